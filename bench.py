@@ -1,0 +1,494 @@
+#!/usr/bin/env python
+"""bench.py — paged KV-migration throughput on B200 (BJ:metric "KV migration GB/s
+(fraction of NVLink/HBM roofline) at 1/2/4/8 B200").
+
+Step = one pass of the hot path over one batch: migrate a whole C2 workload (OPT-13B KV,
+64 requests, ShareGPT-fit lengths 256-2048) from a prefill pool to a decode
+pool through its block tables, all 40 layers, with per-layer completion flags (one
+wind_kv_migrate call = one persistent kernel launch).
+  N = 1 : both pools on cuda:0 (HBM-bound intra-device migration).
+  N > 1 : ranks pair up 2k -> 2k+1; the source rank imports the decode rank's pool (CUDA
+          IPC handles exchanged over a gloo process group) and pushes over NVLink peer
+          stores.  An odd last rank runs the N = 1 step.  Weak scaling: every pair moves
+          its own C2 workload.
+`value` = payload bytes (K+V, all layers, whole blocks; table bytes excluded, reading R14)
+of all ranks / max-over-ranks device time.  Extra scenarios (--scenarios, on by default at
+N = 1) report the other §8(a) rows: layer-streamed hand-off, sequential tables,
+compaction (C5), host swap (C1) — each with its own GB/s and roofline fraction.
+
+--impl reference times the CPU oracle (oracle/, plain C, memcpy per chunk on all host
+cores) on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "KV migration GB/s (fraction of NVLink/HBM roofline) at 1/2/4/8 B200"
+GiB = 1 << 30
+
+
+def load_peaks() -> dict:
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": float(d["hbm_gbs"]), "src": "measured", "sm_max_mhz": d.get("sm_max_mhz")}
+    return {"hbm_gbs": 6650.0, "src": "fallback", "sm_max_mhz": 1965.0}
+
+
+# ------------------------------------------------------------------------ clocks
+
+class ClockSampler:
+    """nvidia-smi sampling DURING the timed region (B200_PROFILING.md clocks line)."""
+
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines: list[str] = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits", "-lms", "50",
+                 "-i", str(self.device)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self._t = threading.Thread(target=self._read, daemon=True)
+            self._t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self) -> dict:
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for n, v in zip(names, f[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------- helpers
+
+def payload_bytes(n_blocks: int, n_layers: int, chunk: int) -> int:
+    """P5 closed form: 2 (K, V) x layers x blocks x C."""
+    return 2 * n_layers * n_blocks * chunk
+
+
+def make_pool(wk, shape, nb, device, seed, tag, loc="device"):
+    import windgen.cuda as wg
+    p = wk.Pool(shape.n_layers, shape.n_kv_heads, shape.head_dim, shape.block_size,
+                shape.elem_bytes, nb, loc=loc, device=device)
+    if loc == "device":
+        wg.fill(p.base, p.nbytes, 0, seed, tag)
+    return p
+
+
+def time_device(fn, steps: int, warmup: int, stream, barrier=None):
+    """W untimed warm-up steps, then EXACTLY `steps` steps between CUDA events on `stream`,
+    barrier + synchronize on both sides.  Returns total ms."""
+    import torch
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    if barrier:
+        barrier()
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(steps):
+        fn()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if barrier:
+        barrier()
+    return e0.elapsed_time(e1)
+
+
+# ------------------------------------------------------------------ cpu baseline
+
+def cpu_baseline(case, n_sample_blocks: int = 160, min_seconds: float = 10.0) -> dict:
+    """The oracle as it stands (or_migrate_mt: T threads memcpy a static partition of the
+    chunk list) on host DRAM pools, bounded sample of the same workload."""
+    import oracle as O
+    sh = case.shape
+    n = min(n_sample_blocks, case.n)
+    nb = math.ceil(1.1 * n)
+    gs = O.Geom(0, sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, nb)
+    src = np.ones(gs.pool_bytes, np.uint8)
+    dst = np.zeros(gs.pool_bytes, np.uint8)
+    sbt = np.random.default_rng(1).permutation(nb)[:n].astype(np.int32)
+    dbt = np.random.default_rng(2).permutation(nb)[:n].astype(np.int32)
+    T = O.hw_threads()
+    O.migrate_mt(src, gs, sbt, dst, gs, dbt, 0, sh.n_layers, T)  # warm (page faults)
+    reps, t0 = 0, time.perf_counter()
+    while True:
+        rc = O.migrate_mt(src, gs, sbt, dst, gs, dbt, 0, sh.n_layers, T)
+        assert rc == O.OK
+        reps += 1
+        el = time.perf_counter() - t0
+        if el >= min_seconds or reps >= 200:
+            break
+    byts = payload_bytes(n, sh.n_layers, sh.chunk_bytes) * reps
+    return {"value": round(byts / el / 1e9, 3), "unit": "GB/s", "cores": T, "kind": "oracle",
+            "sample": f"{n} of {case.n} C2 blocks ({payload_bytes(n, sh.n_layers, sh.chunk_bytes) / GiB:.2f} "
+                      f"GiB payload) x {reps} reps, {el:.1f} s, or_migrate_mt with {T} threads"}
+
+
+def parity_sample(wk, case, src, dst, lo, hi, n_check: int = 96) -> dict:
+    """Sampled bit-exact check of the bench's own output (outside the timed region):
+    the oracle gives each sampled destination chunk's origin (P2 closed form), windgen
+    gives that origin's bytes."""
+    import oracle as O
+    import torch
+    from windgen import content_bytes
+    sh = case.shape
+    gs = O.Geom(0, sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, case.nb_src)
+    gd = O.Geom(0, sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, case.nb_dst)
+    from_src, off = O.expected_origin(gs, case.src_bt, gd, case.dst_bt, lo, hi)
+    rng = np.random.default_rng(7)
+    touched = np.flatnonzero(from_src)
+    idle = np.flatnonzero(from_src == 0)
+    pick = np.concatenate([rng.choice(touched, min(n_check, touched.size), replace=False),
+                           rng.choice(idle, min(n_check // 4, idle.size), replace=False)])
+    C = sh.chunk_bytes
+    t = dst.tensor()
+    bad = 0
+    for c in pick.tolist():
+        got = t[c * C:(c + 1) * C].cpu().numpy()
+        tag = case.src_tag if from_src[c] else case.dst_tag
+        want = content_bytes(case.content_seed, tag, int(off[c]), C)
+        bad += int(not np.array_equal(got, want))
+    torch.cuda.synchronize()
+    return {"chunks_checked": int(pick.size), "mismatches": bad, "ok": bad == 0}
+
+
+# --------------------------------------------------------------------- scenarios
+
+def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
+    """The other §8(a) rows on one GPU, each timed on its own stream with CUDA events."""
+    import torch
+    from windgen import (migration_case, SHAPES, live_mask_after_free, skewed_placement,
+                         request_lengths, blocks_for_tokens)
+    out = {}
+    dev = torch.device("cuda", device)
+    s = torch.cuda.Stream(device)
+    hbm = peaks["hbm_gbs"]
+
+    # (1) C2 sequential tables (long runs: the coalescing / TMA best case)
+    case = migration_case("C2", variant="sequential")
+    sh = case.shape
+    src = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
+    dst = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag)
+    sbt, dbt = torch.as_tensor(case.src_bt, device=dev), torch.as_tensor(case.dst_bt, device=dev)
+    pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
+    ms = time_device(lambda: wk.migrate(src, sbt, dst, dbt, stream=s), steps, warmup, s) / steps
+    gbs = pb / ms / 1e6
+    out["c2_sequential"] = {"gbs": round(gbs, 1), "hbm_frac": round(2 * gbs / hbm, 3), "ms": round(ms, 3)}
+    del src, dst
+
+    # (2) C2 shuffled, layer-streamed hand-off: 40 calls (lo = l, hi = l + 1), a consumer
+    #     stream waits on each layer's flag (A5)
+    case = migration_case("C2")
+    src = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
+    dst = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag)
+    sbt, dbt = torch.as_tensor(case.src_bt, device=dev), torch.as_tensor(case.dst_bt, device=dev)
+    cons = torch.cuda.Stream(device)
+
+    def streamed():
+        for l in range(sh.n_layers):
+            wk.migrate(src, sbt, dst, dbt, layer_lo=l, layer_hi=l + 1, stream=s)
+        t = dst.layer_ticket()
+        for l in range(sh.n_layers):
+            wk.layer_wait(dst, l, t, stream=cons)
+        s.wait_stream(cons)
+    pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
+    ms = time_device(streamed, steps, warmup, s) / steps
+    gbs = pb / ms / 1e6
+    out["c2_layer_streamed"] = {"gbs": round(gbs, 1), "hbm_frac": round(2 * gbs / hbm, 3),
+                                "ms": round(ms, 3), "launches_per_step": sh.n_layers}
+    del src, dst
+
+    # (3) C5 compaction on GPU 0's share of the skewed placement (A7)
+    sh5 = SHAPES["C5"]
+    lens = request_lengths("C5")
+    place = skewed_placement(lens.size, 8, 4005)
+    reqb = blocks_for_tokens(lens[place == 0], 16)
+    nb = math.ceil(int(reqb.sum()) * 1.1)
+    live, _ = live_mask_after_free(nb, reqb, 0.5, 4006)
+    csrc, cdst = wk.plan_compact(live)
+    pool = make_pool(wk, sh5, nb, device, 3005, 1)
+    ts, td = torch.as_tensor(csrc, device=dev), torch.as_tensor(cdst, device=dev)
+    pb = payload_bytes(len(csrc), sh5.n_layers, sh5.chunk_bytes)
+    # compaction is idempotent under repetition only for the first run; moving the same
+    # pairs again re-copies identical bytes (same traffic), which is what is timed
+    ms = time_device(lambda: wk.compact(pool, ts, td, stream=s), steps, warmup, s) / steps
+    gbs = pb / ms / 1e6
+    out["c5_compact"] = {"gbs": round(gbs, 1), "hbm_frac": round(2 * gbs / hbm, 3), "ms": round(ms, 3),
+                         "moves": int(len(csrc)), "pool_gib": round(pool.nbytes / GiB, 2)}
+    del pool
+
+    # (4) C1 host swap round trip over PCIe (A6): swap_out then swap_in at other slots
+    case = migration_case("C1")
+    sh1 = case.shape
+    dpool = make_pool(wk, sh1, case.nb_src, device, case.content_seed, case.src_tag)
+    dpool2 = make_pool(wk, sh1, case.nb_dst, device, case.content_seed, case.dst_tag)
+    hpool = wk.Pool(sh1.n_layers, sh1.n_kv_heads, sh1.head_dim, sh1.block_size, sh1.elem_bytes,
+                    case.n, loc="host")
+    hbt = torch.arange(case.n, dtype=torch.int32, device=dev)
+    sbt, dbt = torch.as_tensor(case.src_bt, device=dev), torch.as_tensor(case.dst_bt, device=dev)
+    pb = payload_bytes(case.n, sh1.n_layers, sh1.chunk_bytes)
+    ms_o = time_device(lambda: wk.swap_out(dpool, sbt, hpool, hbt, stream=s), steps, warmup, s) / steps
+    ms_i = time_device(lambda: wk.swap_in(hpool, hbt, dpool2, dbt, stream=s), steps, warmup, s) / steps
+    pcie = 63.0
+    out["c1_swap"] = {"out_gbs": round(pb / ms_o / 1e6, 2), "in_gbs": round(pb / ms_i / 1e6, 2),
+                      "pcie_gen5_frac_out": round(pb / ms_o / 1e6 / pcie, 3),
+                      "pcie_gen5_frac_in": round(pb / ms_i / 1e6 / pcie, 3),
+                      "payload_mib": round(pb / (1 << 20), 1), "pcie_peak_gbs": pcie}
+    # copy-engine comparator (the practical PCIe ceiling)
+    hbuf = torch.empty(pb, dtype=torch.uint8, pin_memory=True)
+    dbuf = torch.empty(pb, dtype=torch.uint8, device=dev)
+    ms_ce = time_device(lambda: hbuf.copy_(dbuf, non_blocking=True), steps, warmup,
+                        torch.cuda.current_stream(device)) / steps
+    out["c1_swap"]["copy_engine_d2h_gbs"] = round(pb / ms_ce / 1e6, 2)
+    del dpool, dpool2, hpool
+    return out
+
+
+# -------------------------------------------------------------------------- main
+
+def run_gpu(args) -> None:
+    import torch
+    import torch.distributed as dist
+    import paper_conf_isca_fenghzly025_b200 as wk
+    from windgen import migration_case
+
+    rank = int(os.environ.get("RANK", 0))
+    world = int(os.environ.get("WORLD_SIZE", 1))
+    local = int(os.environ.get("LOCAL_RANK", 0))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+    barrier = (lambda: dist.barrier()) if world > 1 else None
+    peaks = load_peaks()
+
+    case = migration_case(args.config, variant=args.variant)
+    sh = case.shape
+    role = "solo"
+    if world > 1:
+        if rank % 2 == 0 and rank + 1 < world:
+            role = "push"
+        elif rank % 2 == 1:
+            role = "decode"
+    src = dst = None
+    if role in ("solo", "push"):
+        src = make_pool(wk, sh, case.nb_src, local, case.content_seed, case.src_tag)
+    if role in ("solo", "decode"):
+        dst = make_pool(wk, sh, case.nb_dst, local, case.content_seed, case.dst_tag)
+    if world > 1:
+        handles = [None] * world
+        dist.all_gather_object(handles, dst.export() if role == "decode" else None)
+        if role == "push":
+            dst = wk.Pool.import_(handles[rank + 1], local)
+    stream = torch.cuda.Stream(local)
+    sbt = torch.as_tensor(case.src_bt, device=dev)
+    dbt = torch.as_tensor(case.dst_bt, device=dev)
+    lo, hi = 0, sh.n_layers
+    pb = payload_bytes(case.n, hi - lo, sh.chunk_bytes)
+
+    def step():
+        if role != "decode":
+            wk.migrate(src, sbt, dst, dbt, layer_lo=lo, layer_hi=hi, stream=stream)
+
+    torch.cuda.synchronize()
+    launches0 = wk.launch_count()
+    with ClockSampler(local) as clk:
+        ms_total = time_device(step, args.steps, args.warmup, stream, barrier)
+    launches = wk.launch_count() - launches0 - (args.warmup if role != "decode" else 0)
+    ms_step_local = ms_total / args.steps
+    # e2e: tables from pinned host memory H2D, the migrate, the layer flags read back D2H
+    h_sbt = torch.as_tensor(case.src_bt).pin_memory()
+    h_dbt = torch.as_tensor(case.dst_bt).pin_memory()
+    d_sbt, d_dbt = torch.empty_like(sbt), torch.empty_like(dbt)
+    flags_host = torch.empty(sh.n_layers, dtype=torch.int32).pin_memory()
+    flags_dev = dst.flags_tensor(local) if dst is not None else None
+
+    def e2e_step():
+        if role == "decode":
+            return
+        with torch.cuda.stream(stream):
+            d_sbt.copy_(h_sbt, non_blocking=True)
+            d_dbt.copy_(h_dbt, non_blocking=True)
+        wk.migrate(src, d_sbt, dst, d_dbt, layer_lo=lo, layer_hi=hi, stream=stream)
+        with torch.cuda.stream(stream):
+            flags_host.copy_(flags_dev, non_blocking=True)
+        stream.synchronize()
+
+    ms_e2e_local = time_device(e2e_step, max(3, args.steps // 2), 2, stream, barrier) / max(3, args.steps // 2)
+
+    # max over ranks
+    t = torch.tensor([ms_step_local, ms_e2e_local], dtype=torch.float64)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    ms_step, ms_e2e = float(t[0]), float(t[1])
+    n_movers = sum(1 for r in range(world) if not (r % 2 == 1) or world == 1) if world > 1 else 1
+    if world > 1:
+        n_movers = world // 2 + (world % 2)
+    total_bytes = pb * n_movers
+    value = total_bytes / ms_step / 1e6  # GB/s
+    e2e_value = total_bytes / ms_e2e / 1e6
+
+    extra = {}
+    if rank == 0:
+        kernel_gbs = pb / ms_step_local / 1e6
+        if role == "solo":
+            roof = {"bound": "hbm", "achieved": round(2 * kernel_gbs, 1), "peak": peaks["hbm_gbs"],
+                    "unit": "GB/s", "frac": round(2 * kernel_gbs / peaks["hbm_gbs"], 4),
+                    "traffic": traffic_from_profiles(args.config), "peak_src": peaks["src"],
+                    "per_launch_bytes": 2 * pb,
+                    "note": "algorithmic DRAM bytes = 2 x payload (read + write) per launch; "
+                            "1 launch (wind_kv tma_copy_kernel) per step"}
+        else:
+            roof = {"bound": "nvlink", "achieved": round(kernel_gbs, 1), "peak": 900.0, "unit": "GB/s",
+                    "frac": round(kernel_gbs / 900.0, 4), "traffic": None, "peak_src": "nominal",
+                    "per_launch_bytes": pb}
+        extra["roofline"] = roof
+        extra["parity"] = parity_sample(wk, case, src, dst, lo, hi) if role == "solo" else None
+        if world == 1 and not args.no_cpu_baseline:
+            extra["cpu_baseline"] = cpu_baseline(case)
+        if world == 1 and args.scenarios:
+            del src, dst
+            torch.cuda.empty_cache()
+            extra["scenarios"] = run_scenarios(wk, local, peaks)
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": "GB/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 4),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "dtype": "u8", "data": "synthetic",
+            "config": {"workload": f"{args.config} {sh.name} KV: {case.n} blocks of {case.lengths.size} "
+                                   f"requests (ShareGPT-fit 256-2048 tok), {args.variant} tables, "
+                                   f"prefill pool -> decode pool, layers 0-{sh.n_layers - 1}",
+                       "payload_gib_per_pair": round(pb / GiB, 3),
+                       "placement": "same GPU" if world == 1 else "pairs 2k->2k+1 over NVLink peer stores",
+                       "l2": "inputs >> 126 MB L2 (no flush needed)",
+                       "parallelism": f"{n_movers} independent mover(s)"},
+            "e2e": {"value": round(e2e_value, 2), "unit": "GB/s",
+                    "h2d_bytes_per_step": int(8 * case.n), "d2h_bytes_per_step": int(4 * sh.n_layers)},
+            "gpu_launches": int(launches),
+            "clocks": clk.summary(),
+            **extra,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+def traffic_from_profiles(cfg: str):
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if not os.path.exists(p):
+        return None
+    try:
+        return json.load(open(p)).get(cfg, {}).get("dram_bytes_per_launch")
+    except Exception:
+        return None
+
+
+def run_reference(args) -> None:
+    """--impl reference: the CPU oracle as it stands on this host's cores, rank 0 only."""
+    rank = int(os.environ.get("RANK", 0))
+    if rank != 0:
+        return
+    import oracle as O
+    from windgen import migration_case
+    case = migration_case(args.config, variant=args.variant)
+    sh = case.shape
+    n = min(64, case.n)  # bounded sample per step
+    nb = math.ceil(1.1 * n)
+    g = O.Geom(0, sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, nb)
+    src = np.ones(g.pool_bytes, np.uint8)
+    dst = np.zeros(g.pool_bytes, np.uint8)
+    sbt = np.random.default_rng(1).permutation(nb)[:n].astype(np.int32)
+    dbt = np.random.default_rng(2).permutation(nb)[:n].astype(np.int32)
+    T = O.hw_threads()
+    for _ in range(args.warmup):
+        O.migrate_mt(src, g, sbt, dst, g, dbt, 0, sh.n_layers, T)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        assert O.migrate_mt(src, g, sbt, dst, g, dbt, 0, sh.n_layers, T) == O.OK
+    el = time.perf_counter() - t0
+    pb = payload_bytes(n, sh.n_layers, sh.chunk_bytes)
+    v = pb * args.steps / el / 1e9
+    sample = f"{n} of {case.n} {args.config} blocks ({pb / GiB:.2f} GiB payload) per step"
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": round(v, 3), "unit": "GB/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": round(el / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": f"{args.config} {sh.name} KV, {args.variant} tables (oracle sample)"},
+        "cpu_baseline": {"value": round(v, 3), "unit": "GB/s", "cores": T, "kind": "oracle",
+                         "sample": sample},
+        "e2e": {"value": round(v, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="wind_kv", choices=["wind_kv", "reference"])
+    ap.add_argument("--config", default="C2")
+    ap.add_argument("--variant", default="shuffled", choices=["shuffled", "sequential"])
+    ap.add_argument("--scenarios", dest="scenarios", action="store_true", default=True)
+    ap.add_argument("--no-scenarios", dest="scenarios", action="store_false")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_gpu(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,264 @@
+/* wind_kv.h — C ABI of the B200-native paged KV-cache migration library.
+ *
+ * The library implements the data-parallel hot path under WindServe's stall-free
+ * rescheduling and KV-swap reduction (Feng et al., ISCA '25; PAPER.md = the paper text,
+ * "P:n" = its line n): a request's K/V blocks are gathered, layer by layer, from a source
+ * block pool through its block table and scattered into slots of a destination pool under
+ * a new block table — within one GPU, to another GPU over NVLink, or to / from pinned
+ * host memory.
+ *
+ *   - KV kept in fixed-size blocks with a per-instance KV manager: §2.1, §3.1
+ *   - prefill->decode KV transfer, overlapped with prefill: §2.2, §1
+ *   - KV swap GPU<->CPU under memory pressure: §2.2, §5.2, §5.4
+ *   - decode->prefill migration of long-context requests (Dynamic Rescheduling) while
+ *     decoding continues (stall-free): §3.2.2, §3.3
+ *   - layers run in sequential order, so KV can be handed over layer by layer: P:219
+ *   - no allocation / implicit stream sync on the hot path: §4
+ * Everything the paper leaves open (layout, aliasing, slot choice, ...) follows the
+ * readings R1-R21 listed in DESIGN.md (= SURVEY.md §8(c) A1-A21).
+ *
+ * Conventions
+ *   - Every function returns wind_status: 0 = OK, < 0 = error.  Nothing throws or aborts
+ *     across the ABI.  wind_kv_last_error() returns detail text (thread-local).
+ *   - Argument errors are detected synchronously, before anything is enqueued, in this
+ *     precedence: INVALID_ARG > GEOMETRY > LAYER_RANGE > NO_PEER.
+ *   - Ops are asynchronous on the given stream, never allocate and never synchronise the
+ *     host; they are CUDA-graph capturable.  Asynchronous CUDA faults surface at
+ *     the caller's next synchronisation, as with any CUDA call.
+ *   - `cudaStream_t` parameters are passed as `void*` (0 = the legacy default stream) so
+ *     the header needs no CUDA include.
+ */
+#ifndef WIND_KV_H
+#define WIND_KV_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef int32_t wind_status;
+
+enum {
+  WIND_OK = 0,
+  WIND_ERR_INVALID_ARG = -1,   /* null handle, n < 0, wrong stream device, misaligned */
+  WIND_ERR_GEOMETRY = -2,      /* H, d, block_size or elem_bytes differ between pools */
+  WIND_ERR_LAYER_RANGE = -3,   /* lo > hi, or [lo, hi) not inside both pools */
+  WIND_ERR_BLOCK_RANGE = -4,   /* a table entry outside [0, n_blocks) */
+  WIND_ERR_DUP_DST = -5,       /* two entries of dst_bt name the same slot */
+  WIND_ERR_ALIAS = -6,         /* same pool: a destination slot is another entry's source */
+  WIND_ERR_NO_PEER = -7,       /* pools on devices that cannot reach each other */
+  WIND_ERR_CUDA = -8,          /* a CUDA runtime / driver call failed (see last_error) */
+  WIND_ERR_OOM = -9,           /* allocation failed (pool create / import only) */
+  WIND_ERR_UNSUPPORTED = -10,  /* geometry the kernels do not support (C % 16 != 0, ...) */
+  WIND_ERR_DEVICE_CHECK = -11  /* debug pools: the device-side table check fired */
+};
+
+typedef enum { WIND_LOC_DEVICE = 0, WIND_LOC_HOST = 1 /* pinned, mapped, portable */ } wind_loc;
+
+/* Pool flags. */
+#define WIND_POOL_DEBUG 0x1u /* ops into/out of this pool also run a device table check */
+
+/* Pool descriptor.  Layout (reading R2): [L][2][NB][H][bs][d] elements of
+ * elem_bytes, layer-major with K/V planes; chunk (layer l, kv, block b) is the C =
+ * H*bs*d*elem_bytes contiguous bytes at offset (((l - first_layer)*2 + kv)*NB + b)*C, and
+ * each head tile (H index h) is the contiguous bs*d*elem_bytes bytes inside it (HND).
+ * Layers are GLOBAL ids [first_layer, first_layer + n_layers) (PP stages).
+ * Requirements: every extent >= 1, n_layers <= WIND_KV_MAX_LAYERS, elem_bytes in {1,2,4}
+ * (fp8 / fp16|bf16 / fp32 payloads are raw bytes, never interpreted: reading R13),
+ * C % 16 == 0.  `device` is ignored for host pools. */
+typedef struct {
+  int32_t first_layer, n_layers;
+  int32_t n_kv_heads, head_dim, block_size, elem_bytes;
+  int32_t n_blocks;
+  int32_t loc;    /* wind_loc */
+  int32_t device; /* CUDA ordinal of a device pool */
+  uint32_t flags; /* WIND_POOL_* */
+} wind_kv_pool_desc;
+
+#define WIND_KV_MAX_LAYERS 1024
+
+typedef struct wind_kv_pool wind_kv_pool; /* opaque */
+
+#define WIND_KV_IPC_HANDLE_BYTES 512
+typedef struct {
+  unsigned char bytes[WIND_KV_IPC_HANDLE_BYTES];
+} wind_kv_ipc_handle;
+
+/* ------------------------------------------------------------------- pools (§8(a) A1) */
+
+/* Creates a pool.  external_base == NULL: the library allocates the data (cudaMalloc on
+ * desc->device, or cudaHostAlloc(Mapped|Portable) for host pools) and frees it on
+ * destroy.  external_base != NULL: the caller's memory (device memory on desc->device, or
+ * mapped pinned host memory for host pools; >= pool bytes; 16-B aligned, else
+ * INVALID_ARG) is used and never freed.  The pool's layer_done flags (one uint32 per
+ * layer, zeroed) are always library-allocated: device memory for device pools, mapped
+ * pinned memory for host pools.  Contents of library-allocated data are undefined.
+ * Errors: INVALID_ARG, UNSUPPORTED, OOM, CUDA.  *out is set only on success. */
+wind_status wind_kv_pool_create(const wind_kv_pool_desc* desc, void* external_base,
+                                wind_kv_pool** out);
+
+/* Destroys a pool handle.  Frees only library-allocated memory; imported pools are only
+ * unmapped.  The caller guarantees no op using the pool is still in flight.  NULL is OK. */
+wind_status wind_kv_pool_destroy(wind_kv_pool* pool);
+
+/* Base address (device-accessible; for host pools the mapped pointer, valid on host and
+ * device under UVA), size in bytes, and descriptor (for imported pools: the owner's
+ * descriptor with `device` = the importing device).  Any out pointer may be NULL. */
+wind_status wind_kv_pool_info(const wind_kv_pool* pool, void** base, size_t* bytes,
+                              wind_kv_pool_desc* desc);
+
+/* Address of the pool's layer_done[n_layers] uint32 flags (device-accessible), for
+ * consumers that poll in their own kernels.  Flag i belongs to global layer
+ * first_layer + i. */
+wind_status wind_kv_pool_flags(const wind_kv_pool* pool, uint32_t** layer_done);
+
+/* Exports a DEVICE pool (data + layer flags) for another process (CUDA IPC).  The handle
+ * is plain bytes: send it over any channel (e.g. a torch process group).  Host pools:
+ * UNSUPPORTED. */
+wind_status wind_kv_pool_export(const wind_kv_pool* pool, wind_kv_ipc_handle* out);
+
+/* Imports an exported pool into this process, mapped for `local_device` (peer access is
+ * enabled from local_device to the owner's device when they differ; NO_PEER if it cannot
+ * be).  The imported pool can be the destination (push, P:120 hand-off) or the source
+ * (pull) of migrate.  Importing in the exporting process itself is UNSUPPORTED (CUDA IPC
+ * restriction). */
+wind_status wind_kv_pool_import(const wind_kv_ipc_handle* handle, int32_t local_device,
+                                wind_kv_pool** out);
+
+/* ------------------------------------------------------------ data movement (A2-A7) */
+
+/* migrate (A2-A5): for every global layer l in [layer_lo, layer_hi), kv in {K, V} and
+ * i in [0, n_blocks):   dst[l][kv][dst_bt[i]] := src_before[l][kv][src_bt[i]]
+ * (C raw bytes).  All other bytes of dst are unchanged (R20).
+ *   src_bt, dst_bt: BORROWED int32[n_blocks], device-accessible from the executing
+ *     device (device memory or mapped pinned host memory); they must stay valid and
+ *     unmodified until the op completes on `stream` (the cudaMemcpyAsync contract).
+ *   Table contract (R4, R5): entries in range, dst_bt pairwise distinct, and if src and
+ *     dst are the same pool, dst_bt[i] == src_bt[j] only for i == j.  Duplicate sources
+ *     (fan-out) are allowed.  Release builds do not check table CONTENT on the hot path
+ *     (use wind_kv_validate, or WIND_POOL_DEBUG pools); violating it leaves dst undefined
+ *     in the affected chunks, never memory outside the two pools' tables' slots.
+ *   Executing device: src's device if src is a device pool (its own, or the device an
+ *     imported src was mapped into), else dst's.  `stream` must belong to it
+ *     (INVALID_ARG otherwise).  Cross-device ops push over NVLink peer stores (or pull
+ *     when src is the remote one); host pools move over PCIe via mapped memory.
+ *   Layer flags (A5): every call with n_blocks > 0 and lo < hi takes one ticket on dst
+ *     (see wind_kv_layer_ticket) and, as each layer's bytes become visible system-wide,
+ *     adds 1 to dst's layer_done flag of that layer; flags of dst layers outside
+ *     [lo, hi) are incremented at the start of the op, so "flag >= ticket" is meaningful
+ *     for every layer.  Layers are processed in ascending order.
+ *   n_blocks == 0 or layer_lo == layer_hi: WIND_OK, nothing enqueued, no ticket (R19). */
+wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind_kv_pool* dst,
+                            const int32_t* dst_bt, int32_t n_blocks, int32_t layer_lo,
+                            int32_t layer_hi, void* stream);
+
+/* swap_out / swap_in (A6): migrate over all layers of the device pool with a HOST pool as
+ * destination / source.  The host pool must cover the device pool's
+ * layers.  Executes on the device pool's GPU; SM stores to / loads from mapped pinned
+ * memory over PCIe. */
+wind_status wind_kv_swap_out(const wind_kv_pool* dev, const int32_t* dev_bt,
+                             wind_kv_pool* host, const int32_t* host_bt, int32_t n_blocks,
+                             void* stream);
+wind_status wind_kv_swap_in(const wind_kv_pool* host, const int32_t* host_bt,
+                            wind_kv_pool* dev, const int32_t* dev_bt, int32_t n_blocks,
+                            void* stream);
+
+/* compact (A7): migrate(pool, src_bt, pool, dst_bt, n, l0, l0 + L) — in-place moves of
+ * live blocks into holes; tables typically from wind_kv_plan_compact. */
+wind_status wind_kv_compact(wind_kv_pool* pool, const int32_t* src_bt, const int32_t* dst_bt,
+                            int32_t n_blocks, void* stream);
+
+/* One entry of a batched migrate: several (dst pool, tables) pairs from ONE source pool,
+ * executed by one persistent launch (all-to-all rebalancing, A8: a GPU pushing to up to
+ * 7 peers at once).  Each entry takes its own ticket on its dst. */
+typedef struct {
+  wind_kv_pool* dst;
+  const int32_t* src_bt;
+  const int32_t* dst_bt;
+  int32_t n_blocks;
+} wind_kv_migrate_item;
+
+#define WIND_KV_MAX_BATCH 16
+
+/* Batched migrate (A8): items[0..n_items) all read from `src`, layers [lo, hi), in one
+ * launch on `stream`.  Destination pools must be pairwise distinct objects with
+ * disjoint memory (the planner guarantees it).  n_items <= WIND_KV_MAX_BATCH. */
+wind_status wind_kv_migrate_batch(const wind_kv_pool* src, const wind_kv_migrate_item* items,
+                                  int32_t n_items, int32_t layer_lo, int32_t layer_hi,
+                                  void* stream);
+
+/* ------------------------------------------------------------- layer flags (A5) */
+
+/* Number of ops this process has enqueued into `dst` so far (the ticket of the latest). */
+wind_status wind_kv_layer_ticket(const wind_kv_pool* dst, uint32_t* ticket);
+
+/* Makes `consumer` wait (device-side, no host sync) until dst's layer_done for global
+ * `layer` reaches `ticket` (wrap-safe >=), i.e. until that many ops have landed that
+ * layer.  Uses cuStreamWaitValue32(GEQ) on the flag, local to dst.  When ops into one
+ * pool are issued on one stream, flag >= t means ops 1..t are complete for that layer. */
+wind_status wind_kv_layer_wait(const wind_kv_pool* dst, int32_t layer, uint32_t ticket,
+                               void* consumer);
+
+/* Host read of layer_done[layer] (synchronous; tests and diagnostics). */
+wind_status wind_kv_layer_count(const wind_kv_pool* dst, int32_t layer, uint32_t* value);
+
+/* --------------------------------------------------------------- host-side logic */
+
+/* Checks an op completely on HOST copies of the tables, O(n): the argument checks of
+ * migrate, then BLOCK_RANGE > DUP_DST > ALIAS, each over the whole table (R4, R5). */
+wind_status wind_kv_validate(const wind_kv_pool* src, const int32_t* src_bt_host,
+                             const wind_kv_pool* dst, const int32_t* dst_bt_host, int32_t n,
+                             int32_t layer_lo, int32_t layer_hi);
+
+/* Compaction plan (A7, two-finger): live[n_slots] (0/1).  With n_live = sum(live):
+ * holes = ascending b < n_live with !live[b]; movers = ascending b >= n_live with
+ * live[b]; pair k moves movers[k] -> holes[k].  Writes n_moves entries to src_bt/dst_bt
+ * (caller buffers of n_slots entries).  The pairs satisfy the same-pool table contract. */
+wind_status wind_kv_plan_compact(const uint8_t* live, int32_t n_slots, int32_t* src_bt,
+                                 int32_t* dst_bt, int32_t* n_moves);
+
+/* Rebalance plan (A8, greedy; not in the paper — nearest P:219-227):
+ * target = ceil(sum blocks / G); repeat { src = most loaded GPU, dst = least loaded
+ * (lowest id on ties); stop if load[src] <= target; move the longest request of src that
+ * keeps dst <= target (lowest id on ties; longest-first per P:227); stop if none }.
+ * out_gpu[r] = final GPU of request r. */
+wind_status wind_kv_plan_rebalance(int32_t n_gpus, int32_t n_requests, const int32_t* req_gpu,
+                                   const int32_t* req_blocks, int32_t* out_gpu,
+                                   int32_t* n_moves);
+
+/* Debug pools: synchronises the pool's device and returns DEVICE_CHECK if a device-side
+ * table check recorded an error (then clears it), else OK. */
+wind_status wind_kv_check_device_error(const wind_kv_pool* pool);
+
+/* ------------------------------------------------------------------ tuning & misc */
+
+/* Kernel selection and launch shape, per path.  Defaults are the measured best on B200
+ * (DESIGN.md §Kernels).  kernel: 0 = auto, 1 = TMA bulk staged copy, 2 = SIMT 16-B
+ * vector copy.  ctas_per_sm, stage_bytes (TMA stage / SIMT unit bytes, multiple of 16),
+ * stages (TMA ring depth); 0 keeps the current value. */
+typedef enum { WIND_PATH_INTRA = 0, WIND_PATH_PEER = 1, WIND_PATH_HOST = 2 } wind_path;
+typedef struct {
+  int32_t kernel;
+  int32_t ctas_per_sm;
+  int32_t stage_bytes;
+  int32_t stages;
+  int32_t max_ctas; /* cap on the grid (e.g. to leave SMs to a decode stream); 0 = none */
+  int32_t evict_first; /* 1 = L2 evict-first policy on the copy's loads and stores */
+} wind_kv_tuning;
+
+wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t);
+wind_status wind_kv_get_tuning(int32_t path, wind_kv_tuning* t);
+
+/* Number of kernels this process has launched through the library (all ops). */
+uint64_t wind_kv_launch_count(void);
+
+const char* wind_kv_status_string(wind_status s);
+const char* wind_kv_last_error(void);
+const char* wind_kv_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* WIND_KV_H */

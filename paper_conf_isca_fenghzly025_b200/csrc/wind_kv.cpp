@@ -1,0 +1,855 @@
+// wind_kv.cpp — host side of the C ABI (include/wind_kv.h): pools and peer mapping,
+// argument checking, table validation, planners, tickets / layer waits, and the launch of
+// the copy kernels (wind_kv_kernels.cu).  No allocation and no host synchronisation on the
+// migrate / swap / compact path: everything an op needs (layer
+// flags, arrival-counter ring) is allocated when a pool is created or imported.
+#include <cuda.h>
+#include <cuda_runtime.h>
+#include <stdarg.h>
+#include <stdint.h>
+#include <stdio.h>
+#include <string.h>
+#include <unistd.h>
+
+#include <algorithm>
+#include <atomic>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "wind_kv_internal.h"
+
+using namespace wkv;
+
+// --------------------------------------------------------------------------- errors
+
+namespace {
+
+thread_local std::string g_last_error;
+std::atomic<uint64_t> g_launches{0};
+
+wind_status fail(wind_status code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_last_error = buf;
+  return code;
+}
+
+wind_status cuda_fail(cudaError_t e, const char* what) {
+  return fail(WIND_ERR_CUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+#define WKV_CUDA(call, what)                        \
+  do {                                              \
+    cudaError_t _e = (call);                        \
+    if (_e != cudaSuccess) return cuda_fail(_e, what); \
+  } while (0)
+
+// Restores the caller's current device on scope exit.
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    cudaGetDevice(&prev);
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int now = -1;
+    cudaGetDevice(&now);
+    if (prev >= 0 && now != prev) cudaSetDevice(prev);
+  }
+};
+
+// ------------------------------------------------------------- driver entry points
+
+typedef CUresult (*PFN_waitValue32)(CUstream, CUdeviceptr, cuuint32_t, unsigned int);
+typedef CUresult (*PFN_getAddressRange)(CUdeviceptr*, size_t*, CUdeviceptr);
+
+template <typename F>
+F driver_fn(const char* name) {
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPointByVersion(name, &fn, 12000, cudaEnableDefault, &q) != cudaSuccess ||
+      q != cudaDriverEntryPointSuccess)
+    return nullptr;
+  return reinterpret_cast<F>(fn);
+}
+
+// ------------------------------------------------------------ per-device context
+
+struct DevCtx {
+  std::mutex mu;
+  bool ready = false;
+  int sms = 0;
+  uint8_t uuid[16] = {};
+  uint32_t* counters = nullptr;  // kCounterSlots * WIND_KV_MAX_LAYERS, zeroed
+  std::atomic<uint64_t> seq{0};
+  size_t tma_smem_set = 0;
+  int32_t* err = nullptr;        // debug device-check word
+  uint32_t* scratch = nullptr;   // debug table-check scratch
+  int32_t scratch_n = 0;
+};
+
+constexpr int kMaxDevices = 64;
+DevCtx g_dev[kMaxDevices];
+
+wind_status dev_ctx(int dev, DevCtx** out) {
+  if (dev < 0 || dev >= kMaxDevices) return fail(WIND_ERR_INVALID_ARG, "device %d out of range", dev);
+  DevCtx& c = g_dev[dev];
+  std::lock_guard<std::mutex> lk(c.mu);
+  if (!c.ready) {
+    int n = 0;
+    WKV_CUDA(cudaGetDeviceCount(&n), "cudaGetDeviceCount");
+    if (dev >= n) return fail(WIND_ERR_INVALID_ARG, "device %d not present (%d devices)", dev, n);
+    DeviceGuard g(dev);
+    cudaDeviceProp prop;
+    WKV_CUDA(cudaGetDeviceProperties(&prop, dev), "cudaGetDeviceProperties");
+    c.sms = prop.multiProcessorCount;
+    memcpy(c.uuid, &prop.uuid, 16);
+    const size_t cbytes = sizeof(uint32_t) * kCounterSlots * WIND_KV_MAX_LAYERS;
+    WKV_CUDA(cudaMalloc(&c.counters, cbytes), "cudaMalloc(counters)");
+    WKV_CUDA(cudaMemset(c.counters, 0, cbytes), "cudaMemset(counters)");
+    WKV_CUDA(cudaMalloc(&c.err, sizeof(int32_t)), "cudaMalloc(err)");
+    WKV_CUDA(cudaMemset(c.err, 0, sizeof(int32_t)), "cudaMemset(err)");
+    const size_t max_smem = 227 * 1024;
+    WKV_CUDA(prepare_kernels(dev, max_smem), "cudaFuncSetAttribute(tma smem)");
+    c.tma_smem_set = max_smem;
+    c.ready = true;
+  }
+  *out = &c;
+  return WIND_OK;
+}
+
+// ------------------------------------------------------------------------- tuning
+
+std::mutex g_tune_mu;
+wind_kv_tuning g_tune[3] = {
+    /* INTRA */ {kTma, 1, 32768, 6, 0, 0},
+    /* PEER  */ {kSimt, 4, 32768, 6, 0, 0},
+    /* HOST  */ {kSimt, 4, 32768, 6, 0, 0},
+};
+
+}  // namespace
+
+// ---------------------------------------------------------------------------- pool
+
+struct wind_kv_pool {
+  wind_kv_pool_desc desc;
+  uint8_t* base = nullptr;    // device-accessible data address
+  size_t bytes = 0;
+  int64_t chunk = 0;          // C
+  uint32_t* flags = nullptr;  // layer_done[n_layers], device-accessible
+  bool owns_data = false, owns_flags = false, imported = false;
+  void* ipc_data_base = nullptr;   // imported: mapping to close
+  void* ipc_flags_base = nullptr;
+  uint8_t uuid[16] = {};           // physical GPU of the memory (device pools)
+  std::atomic<uint32_t> enqueued{0};
+};
+
+namespace {
+
+int64_t chunk_bytes_of(const wind_kv_pool_desc& d) {
+  return static_cast<int64_t>(d.n_kv_heads) * d.block_size * d.head_dim * d.elem_bytes;
+}
+
+wind_status check_desc(const wind_kv_pool_desc* d) {
+  if (!d) return fail(WIND_ERR_INVALID_ARG, "desc is NULL");
+  if (d->n_layers < 1 || d->n_kv_heads < 1 || d->head_dim < 1 || d->block_size < 1 ||
+      d->n_blocks < 1 || d->first_layer < 0)
+    return fail(WIND_ERR_INVALID_ARG, "pool extents must be >= 1 (first_layer >= 0)");
+  if (d->loc != WIND_LOC_DEVICE && d->loc != WIND_LOC_HOST)
+    return fail(WIND_ERR_INVALID_ARG, "loc must be WIND_LOC_DEVICE or WIND_LOC_HOST");
+  if (d->n_layers > WIND_KV_MAX_LAYERS)
+    return fail(WIND_ERR_UNSUPPORTED, "n_layers %d > WIND_KV_MAX_LAYERS", d->n_layers);
+  if (d->elem_bytes != 1 && d->elem_bytes != 2 && d->elem_bytes != 4)
+    return fail(WIND_ERR_UNSUPPORTED, "elem_bytes must be 1, 2 or 4");
+  if (chunk_bytes_of(*d) % 16 != 0)
+    return fail(WIND_ERR_UNSUPPORTED, "chunk bytes H*bs*d*e_b = %lld not a multiple of 16",
+                static_cast<long long>(chunk_bytes_of(*d)));
+  return WIND_OK;
+}
+
+}  // namespace
+
+extern "C" wind_status wind_kv_pool_create(const wind_kv_pool_desc* desc, void* external_base,
+                                           wind_kv_pool** out) {
+  if (!out) return fail(WIND_ERR_INVALID_ARG, "out is NULL");
+  wind_status st = check_desc(desc);
+  if (st != WIND_OK) return st;
+  if (external_base && (reinterpret_cast<uintptr_t>(external_base) & 15))
+    return fail(WIND_ERR_INVALID_ARG, "external_base must be 16-byte aligned");
+  auto* p = new wind_kv_pool();
+  p->desc = *desc;
+  p->chunk = chunk_bytes_of(*desc);
+  p->bytes = static_cast<size_t>(desc->n_layers) * 2 * desc->n_blocks * p->chunk;
+  const size_t fbytes = sizeof(uint32_t) * desc->n_layers;
+  cudaError_t e = cudaSuccess;
+  if (desc->loc == WIND_LOC_DEVICE) {
+    DevCtx* ctx;
+    if ((st = dev_ctx(desc->device, &ctx)) != WIND_OK) { delete p; return st; }
+    memcpy(p->uuid, ctx->uuid, 16);
+    DeviceGuard g(desc->device);
+    if (external_base) {
+      cudaPointerAttributes a;
+      if (cudaPointerGetAttributes(&a, external_base) != cudaSuccess || a.type != cudaMemoryTypeDevice ||
+          a.device != desc->device) {
+        cudaGetLastError();
+        delete p;
+        return fail(WIND_ERR_INVALID_ARG, "external_base is not device memory of device %d", desc->device);
+      }
+      p->base = static_cast<uint8_t*>(external_base);
+    } else {
+      e = cudaMalloc(&p->base, p->bytes);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        delete p;
+        return fail(WIND_ERR_OOM, "cudaMalloc(%zu) failed: %s", p->bytes, cudaGetErrorString(e));
+      }
+      p->owns_data = true;
+    }
+    e = cudaMalloc(&p->flags, fbytes);
+    if (e == cudaSuccess) e = cudaMemset(p->flags, 0, fbytes);
+  } else {
+    if (external_base) {
+      void* dptr = nullptr;
+      if (cudaHostGetDevicePointer(&dptr, external_base, 0) != cudaSuccess) {
+        cudaGetLastError();
+        delete p;
+        return fail(WIND_ERR_INVALID_ARG, "external_base is not mapped pinned host memory");
+      }
+      p->base = static_cast<uint8_t*>(dptr);
+    } else {
+      void* h = nullptr;
+      e = cudaHostAlloc(&h, p->bytes, cudaHostAllocMapped | cudaHostAllocPortable);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        delete p;
+        return fail(WIND_ERR_OOM, "cudaHostAlloc(%zu) failed: %s", p->bytes, cudaGetErrorString(e));
+      }
+      void* dptr = nullptr;
+      cudaHostGetDevicePointer(&dptr, h, 0);
+      p->base = static_cast<uint8_t*>(dptr ? dptr : h);
+      p->owns_data = true;
+    }
+    void* hf = nullptr;
+    e = cudaHostAlloc(&hf, fbytes, cudaHostAllocMapped | cudaHostAllocPortable);
+    if (e == cudaSuccess) {
+      memset(hf, 0, fbytes);
+      void* df = nullptr;
+      cudaHostGetDevicePointer(&df, hf, 0);
+      p->flags = static_cast<uint32_t*>(df ? df : hf);
+    }
+  }
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    p->owns_flags = false;
+    wind_kv_pool_destroy(p);
+    return fail(WIND_ERR_OOM, "layer flag allocation failed: %s", cudaGetErrorString(e));
+  }
+  p->owns_flags = true;
+  *out = p;
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_pool_destroy(wind_kv_pool* p) {
+  if (!p) return WIND_OK;
+  if (p->imported) {
+    DeviceGuard g(p->desc.device);
+    if (p->ipc_data_base) cudaIpcCloseMemHandle(p->ipc_data_base);
+    if (p->ipc_flags_base) cudaIpcCloseMemHandle(p->ipc_flags_base);
+  } else if (p->desc.loc == WIND_LOC_DEVICE) {
+    DeviceGuard g(p->desc.device);
+    if (p->owns_data && p->base) cudaFree(p->base);
+    if (p->owns_flags && p->flags) cudaFree(p->flags);
+  } else {
+    if (p->owns_data && p->base) cudaFreeHost(p->base);
+    if (p->owns_flags && p->flags) cudaFreeHost(p->flags);
+  }
+  cudaGetLastError();
+  delete p;
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_pool_info(const wind_kv_pool* p, void** base, size_t* bytes,
+                                         wind_kv_pool_desc* desc) {
+  if (!p) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
+  if (base) *base = p->base;
+  if (bytes) *bytes = p->bytes;
+  if (desc) *desc = p->desc;
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_pool_flags(const wind_kv_pool* p, uint32_t** layer_done) {
+  if (!p || !layer_done) return fail(WIND_ERR_INVALID_ARG, "NULL argument");
+  *layer_done = p->flags;
+  return WIND_OK;
+}
+
+// ----------------------------------------------------------------------------- IPC
+
+namespace {
+
+constexpr char kMagic[8] = {'W', 'I', 'N', 'D', 'K', 'V', '0', '1'};
+
+struct IpcBlob {
+  char magic[8];
+  int32_t owner_pid;
+  int32_t pad;
+  wind_kv_pool_desc desc;
+  cudaIpcMemHandle_t data;
+  uint64_t data_off;
+  cudaIpcMemHandle_t flags;
+  uint64_t flags_off;
+  uint64_t bytes;
+  uint8_t uuid[16];
+};
+static_assert(sizeof(IpcBlob) <= WIND_KV_IPC_HANDLE_BYTES, "IPC blob too large");
+
+wind_status alloc_base(void* p, void** base) {
+  static PFN_getAddressRange fn = driver_fn<PFN_getAddressRange>("cuMemGetAddressRange");
+  if (!fn) return fail(WIND_ERR_CUDA, "cuMemGetAddressRange entry point unavailable");
+  CUdeviceptr b = 0;
+  size_t sz = 0;
+  if (fn(&b, &sz, reinterpret_cast<CUdeviceptr>(p)) != CUDA_SUCCESS)
+    return fail(WIND_ERR_CUDA, "cuMemGetAddressRange failed");
+  *base = reinterpret_cast<void*>(b);
+  return WIND_OK;
+}
+
+}  // namespace
+
+extern "C" wind_status wind_kv_pool_export(const wind_kv_pool* p, wind_kv_ipc_handle* out) {
+  if (!p || !out) return fail(WIND_ERR_INVALID_ARG, "NULL argument");
+  if (p->desc.loc != WIND_LOC_DEVICE || p->imported)
+    return fail(WIND_ERR_UNSUPPORTED, "only this process's device pools can be exported");
+  DeviceGuard g(p->desc.device);
+  IpcBlob b;
+  memset(&b, 0, sizeof b);
+  memcpy(b.magic, kMagic, 8);
+  b.owner_pid = static_cast<int32_t>(getpid());
+  b.desc = p->desc;
+  b.bytes = p->bytes;
+  memcpy(b.uuid, p->uuid, 16);
+  void* db = nullptr;
+  void* fb = nullptr;
+  wind_status st;
+  if ((st = alloc_base(p->base, &db)) != WIND_OK) return st;
+  if ((st = alloc_base(p->flags, &fb)) != WIND_OK) return st;
+  b.data_off = static_cast<uint64_t>(p->base - static_cast<uint8_t*>(db));
+  b.flags_off = static_cast<uint64_t>(reinterpret_cast<uint8_t*>(p->flags) - static_cast<uint8_t*>(fb));
+  WKV_CUDA(cudaIpcGetMemHandle(&b.data, db), "cudaIpcGetMemHandle(data)");
+  WKV_CUDA(cudaIpcGetMemHandle(&b.flags, fb), "cudaIpcGetMemHandle(flags)");
+  memset(out, 0, sizeof *out);
+  memcpy(out->bytes, &b, sizeof b);
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_pool_import(const wind_kv_ipc_handle* h, int32_t local_device,
+                                           wind_kv_pool** out) {
+  if (!h || !out) return fail(WIND_ERR_INVALID_ARG, "NULL argument");
+  IpcBlob b;
+  memcpy(&b, h->bytes, sizeof b);
+  if (memcmp(b.magic, kMagic, 8) != 0) return fail(WIND_ERR_INVALID_ARG, "not a wind_kv IPC handle");
+  if (b.owner_pid == static_cast<int32_t>(getpid()))
+    return fail(WIND_ERR_UNSUPPORTED, "cannot import a pool in the process that exported it");
+  DevCtx* ctx;
+  wind_status st = dev_ctx(local_device, &ctx);
+  if (st != WIND_OK) return st;
+  DeviceGuard g(local_device);
+  void* db = nullptr;
+  void* fb = nullptr;
+  cudaError_t e = cudaIpcOpenMemHandle(&db, b.data, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    if (e == cudaErrorPeerAccessUnsupported || e == cudaErrorInvalidDevice)
+      return fail(WIND_ERR_NO_PEER, "cannot map the peer pool on device %d: %s", local_device,
+                  cudaGetErrorString(e));
+    return cuda_fail(e, "cudaIpcOpenMemHandle(data)");
+  }
+  e = cudaIpcOpenMemHandle(&fb, b.flags, cudaIpcMemLazyEnablePeerAccess);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    cudaIpcCloseMemHandle(db);
+    return cuda_fail(e, "cudaIpcOpenMemHandle(flags)");
+  }
+  auto* p = new wind_kv_pool();
+  p->desc = b.desc;
+  p->desc.device = local_device;
+  p->chunk = chunk_bytes_of(b.desc);
+  p->bytes = b.bytes;
+  p->base = static_cast<uint8_t*>(db) + b.data_off;
+  p->flags = reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(fb) + b.flags_off);
+  p->imported = true;
+  p->ipc_data_base = db;
+  p->ipc_flags_base = fb;
+  memcpy(p->uuid, b.uuid, 16);
+  *out = p;
+  return WIND_OK;
+}
+
+// ------------------------------------------------------------------ op validation
+
+namespace {
+
+bool same_geometry(const wind_kv_pool_desc& a, const wind_kv_pool_desc& b) {
+  return a.n_kv_heads == b.n_kv_heads && a.head_dim == b.head_dim &&
+         a.block_size == b.block_size && a.elem_bytes == b.elem_bytes;
+}
+
+bool layers_inside(const wind_kv_pool_desc& d, int32_t lo, int32_t hi) {
+  return lo >= d.first_layer && hi <= d.first_layer + d.n_layers;
+}
+
+// Table content checks on host copies, O(n): BLOCK_RANGE > DUP_DST > ALIAS, each over the
+// whole table (R4, R5).
+wind_status check_tables_host(const wind_kv_pool* src, const int32_t* sbt,
+                              const wind_kv_pool* dst, const int32_t* dbt, int32_t n) {
+  const int32_t nbs = src->desc.n_blocks, nbd = dst->desc.n_blocks;
+  for (int32_t i = 0; i < n; ++i)
+    if (static_cast<uint32_t>(sbt[i]) >= static_cast<uint32_t>(nbs) ||
+        static_cast<uint32_t>(dbt[i]) >= static_cast<uint32_t>(nbd))
+      return fail(WIND_ERR_BLOCK_RANGE, "table entry %d out of range (src %d of %d, dst %d of %d)",
+                  i, sbt[i], nbs, dbt[i], nbd);
+  std::vector<uint8_t> hit(static_cast<size_t>(nbd), 0);
+  for (int32_t i = 0; i < n; ++i) {
+    if (hit[dbt[i]]) return fail(WIND_ERR_DUP_DST, "destination slot %d appears twice", dbt[i]);
+    hit[dbt[i]] = 1;
+  }
+  if (src->base == dst->base) {
+    // slot b is a source of some entry j and the destination of some entry i != j
+    std::vector<int32_t> src_of(static_cast<size_t>(nbs), -1);  // an entry using b as source
+    std::vector<uint8_t> multi(static_cast<size_t>(nbs), 0);    // >= 2 entries use it
+    for (int32_t j = 0; j < n; ++j) {
+      if (src_of[sbt[j]] >= 0) multi[sbt[j]] = 1;
+      else src_of[sbt[j]] = j;
+    }
+    for (int32_t i = 0; i < n; ++i) {
+      const int32_t b = dbt[i];
+      if (src_of[b] < 0) continue;
+      if (multi[b] || src_of[b] != i)
+        return fail(WIND_ERR_ALIAS, "same pool: slot %d is written by entry %d and read by another entry", b, i);
+    }
+  }
+  return WIND_OK;
+}
+
+// Argument checks shared by every op: INVALID_ARG > GEOMETRY > LAYER_RANGE.
+wind_status check_args(const wind_kv_pool* src, const wind_kv_pool* dst, int32_t n, int32_t lo,
+                       int32_t hi) {
+  if (!src || !dst) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
+  if (n < 0) return fail(WIND_ERR_INVALID_ARG, "n_blocks < 0");
+  if (!same_geometry(src->desc, dst->desc))
+    return fail(WIND_ERR_GEOMETRY, "pools differ in H/d/block_size/elem_bytes");
+  if (lo > hi) return fail(WIND_ERR_LAYER_RANGE, "layer_lo %d > layer_hi %d", lo, hi);
+  if (lo < hi && (!layers_inside(src->desc, lo, hi) || !layers_inside(dst->desc, lo, hi)))
+    return fail(WIND_ERR_LAYER_RANGE, "layers [%d, %d) not inside both pools", lo, hi);
+  return WIND_OK;
+}
+
+// Which device runs the op, and which tuning path applies.
+wind_status route(const wind_kv_pool* src, const wind_kv_pool* dst, int* exec, int* path) {
+  const bool sd = src->desc.loc == WIND_LOC_DEVICE, dd = dst->desc.loc == WIND_LOC_DEVICE;
+  if (!sd && !dd) return fail(WIND_ERR_UNSUPPORTED, "host -> host migration has no executing device");
+  *exec = sd ? src->desc.device : dst->desc.device;
+  if (!sd || !dd) {
+    *path = WIND_PATH_HOST;
+    return WIND_OK;
+  }
+  const bool same_gpu = memcmp(src->uuid, dst->uuid, 16) == 0;
+  *path = same_gpu ? WIND_PATH_INTRA : WIND_PATH_PEER;
+  if (!src->imported && !dst->imported && src->desc.device != dst->desc.device) {
+    int can = 0;
+    cudaDeviceCanAccessPeer(&can, src->desc.device, dst->desc.device);
+    if (!can) return fail(WIND_ERR_NO_PEER, "device %d cannot access device %d", src->desc.device,
+                          dst->desc.device);
+    DeviceGuard g(src->desc.device);
+    cudaError_t e = cudaDeviceEnablePeerAccess(dst->desc.device, 0);  // once per pair
+    if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_fail(e, "cudaDeviceEnablePeerAccess");
+    cudaGetLastError();
+  }
+  if (src->imported && dst->imported)
+    return fail(WIND_ERR_UNSUPPORTED, "at least one pool must be local to this process");
+  return WIND_OK;
+}
+
+wind_status check_stream(void* stream, int exec) {
+  if (!stream) return WIND_OK;  // legacy default stream of the executing device
+  int sd = -1;
+  cudaError_t e = cudaStreamGetDevice(static_cast<cudaStream_t>(stream), &sd);
+  if (e != cudaSuccess) {
+    cudaGetLastError();
+    return fail(WIND_ERR_INVALID_ARG, "invalid stream: %s", cudaGetErrorString(e));
+  }
+  if (sd != exec) return fail(WIND_ERR_INVALID_ARG, "stream belongs to device %d, op executes on %d", sd, exec);
+  return WIND_OK;
+}
+
+struct OpItem {
+  wind_kv_pool* dst;
+  const int32_t* sbt;
+  const int32_t* dbt;
+  int32_t n;
+};
+
+// Debug pools: device-side table check (not on the release hot path; may allocate scratch).
+wind_status debug_check(DevCtx* ctx, int exec, const wind_kv_pool* src, const OpItem& it,
+                        cudaStream_t s) {
+  const int32_t need = std::max(src->desc.n_blocks, it.dst->desc.n_blocks);
+  if (ctx->scratch_n < need) {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    if (ctx->scratch_n < need) {
+      DeviceGuard g(exec);
+      if (ctx->scratch) cudaFree(ctx->scratch);
+      ctx->scratch = nullptr;
+      ctx->scratch_n = 0;
+      WKV_CUDA(cudaMalloc(&ctx->scratch, sizeof(uint32_t) * 2 * need), "cudaMalloc(debug scratch)");
+      ctx->scratch_n = need;
+    }
+  }
+  WKV_CUDA(launch_table_check(it.sbt, it.dbt, it.n, src->desc.n_blocks, it.dst->desc.n_blocks,
+                              src->base == it.dst->base, ctx->scratch, ctx->scratch_n, ctx->err, s),
+           "table check launch");
+  g_launches += 2;
+  return WIND_OK;
+}
+
+// The common op: src -> items[] over layers [lo, hi) on `stream`.
+wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
+                   int32_t hi, void* stream) {
+  if (!src) return fail(WIND_ERR_INVALID_ARG, "src pool is NULL");
+  if (n_items < 1 || n_items > WIND_KV_MAX_BATCH) return fail(WIND_ERR_INVALID_ARG, "n_items out of range");
+  int exec = -1, path = 0;
+  wind_status st;
+  for (int j = 0; j < n_items; ++j) {
+    if ((st = check_args(src, items[j].dst, items[j].n, lo, hi)) != WIND_OK) return st;
+    if (items[j].n > 0 && (!items[j].sbt || !items[j].dbt)) return fail(WIND_ERR_INVALID_ARG, "block table is NULL");
+    for (int k = 0; k < j; ++k)
+      if (items[k].dst == items[j].dst) return fail(WIND_ERR_INVALID_ARG, "batch destinations must be distinct");
+  }
+  for (int j = 0; j < n_items; ++j) {
+    int e2 = -1, p2 = 0;
+    if ((st = route(src, items[j].dst, &e2, &p2)) != WIND_OK) return st;
+    if (j == 0) { exec = e2; path = p2; }
+    else if (e2 != exec) return fail(WIND_ERR_INVALID_ARG, "batch items execute on different devices");
+    else path = std::max(path, p2);
+  }
+  if ((st = check_stream(stream, exec)) != WIND_OK) return st;
+  int64_t total_n = 0;
+  for (int j = 0; j < n_items; ++j) total_n += items[j].n;
+  if (lo == hi || total_n == 0) return WIND_OK;  // R19: successful no-op, no ticket
+
+  DevCtx* ctx;
+  if ((st = dev_ctx(exec, &ctx)) != WIND_OK) return st;
+  wind_kv_tuning t;
+  {
+    std::lock_guard<std::mutex> lk(g_tune_mu);
+    t = g_tune[path];
+  }
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  DeviceGuard g(exec);
+
+  bool debug = false;
+  for (int j = 0; j < n_items; ++j)
+    if (items[j].n > 0 && ((src->desc.flags | items[j].dst->desc.flags) & WIND_POOL_DEBUG)) {
+      if ((st = debug_check(ctx, exec, src, items[j], s)) != WIND_OK) return st;
+      debug = true;
+    }
+
+  Params p;
+  memset(&p, 0, sizeof p);
+  const int64_t C = src->chunk;
+  const int64_t unit = t.stage_bytes;
+  p.chunk = C;
+  if (C >= unit) {
+    p.parts = static_cast<int32_t>((C + unit - 1) / unit);
+    p.part_bytes = static_cast<int32_t>((((C + p.parts - 1) / p.parts) + 15) / 16 * 16);
+    p.group = 1;
+  } else {
+    p.parts = 1;
+    p.part_bytes = static_cast<int32_t>(C);
+    p.group = static_cast<int32_t>(std::min<int64_t>(kMaxSegs, unit / C));
+  }
+  p.layer_lo = lo;
+  p.n_layers = hi - lo;
+  p.src_plane0 = src->base + static_cast<int64_t>(lo - src->desc.first_layer) * 2 * src->desc.n_blocks * C;
+  p.s_plane_stride = static_cast<int64_t>(src->desc.n_blocks) * C;
+  p.evict_first = t.evict_first;
+  p.stages = t.stages;
+  p.stage_bytes = t.stage_bytes;
+  int32_t base_units = 0;
+  int ni = 0;
+  for (int j = 0; j < n_items; ++j) {
+    const OpItem& it = items[j];  // n == 0 items stay: they take a ticket, bump flags
+    const wind_kv_pool* d = it.dst;
+    Item& q = p.items[ni++];
+    q.sbt = it.sbt;
+    q.dbt = it.dbt;
+    q.n = it.n;
+    q.dst_plane0 = d->base + static_cast<int64_t>(lo - d->desc.first_layer) * 2 * d->desc.n_blocks * C;
+    q.d_plane_stride = static_cast<int64_t>(d->desc.n_blocks) * C;
+    q.flags = d->flags;
+    q.d_flag_lo = lo - d->desc.first_layer;
+    q.d_layers = d->desc.n_layers;
+    q.host_flags = d->desc.loc == WIND_LOC_HOST;
+    const int64_t u = p.parts > 1 ? static_cast<int64_t>(it.n) * p.parts
+                                  : (static_cast<int64_t>(it.n) + p.group - 1) / p.group;
+    if (u + base_units > INT32_MAX) return fail(WIND_ERR_UNSUPPORTED, "too many work units");
+    q.units = static_cast<int32_t>(u);
+    q.unit_base = base_units;
+    base_units += q.units;
+  }
+  p.n_items = ni;
+  p.units_per_plane = base_units;
+  p.total_units = static_cast<int64_t>(2) * p.n_layers * base_units;
+  const uint64_t slot = ctx->seq.fetch_add(1) % kCounterSlots;
+  p.counters = ctx->counters + slot * WIND_KV_MAX_LAYERS;
+  p.abort_word = debug ? ctx->err : nullptr;
+
+  int kernel = t.kernel == kAuto ? (path == WIND_PATH_INTRA ? kTma : kSimt) : t.kernel;
+  int64_t grid = static_cast<int64_t>(ctx->sms) * std::max(1, t.ctas_per_sm);
+  if (t.max_ctas > 0) grid = std::min<int64_t>(grid, t.max_ctas);
+  grid = std::max<int64_t>(1, std::min<int64_t>(grid, p.total_units));
+  cudaError_t e = launch_copy(p, kernel, static_cast<int>(grid), s);
+  if (e != cudaSuccess) return cuda_fail(e, "copy kernel launch");
+  g_launches += 1;
+  for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
+  return WIND_OK;
+}
+
+}  // namespace
+
+// ---------------------------------------------------------------- data-movement ABI
+
+extern "C" wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt,
+                                       wind_kv_pool* dst, const int32_t* dst_bt, int32_t n_blocks,
+                                       int32_t layer_lo, int32_t layer_hi, void* stream) {
+  if (!dst) return fail(WIND_ERR_INVALID_ARG, "dst pool is NULL");
+  OpItem it{dst, src_bt, dst_bt, n_blocks};
+  return run_op(src, &it, 1, layer_lo, layer_hi, stream);
+}
+
+extern "C" wind_status wind_kv_migrate_batch(const wind_kv_pool* src, const wind_kv_migrate_item* items,
+                                             int32_t n_items, int32_t layer_lo, int32_t layer_hi,
+                                             void* stream) {
+  if (!items || n_items < 1 || n_items > WIND_KV_MAX_BATCH)
+    return fail(WIND_ERR_INVALID_ARG, "items NULL or n_items out of [1, %d]", WIND_KV_MAX_BATCH);
+  OpItem its[WIND_KV_MAX_BATCH];
+  for (int j = 0; j < n_items; ++j) {
+    if (!items[j].dst) return fail(WIND_ERR_INVALID_ARG, "batch item %d has no dst", j);
+    its[j] = OpItem{items[j].dst, items[j].src_bt, items[j].dst_bt, items[j].n_blocks};
+  }
+  return run_op(src, its, n_items, layer_lo, layer_hi, stream);
+}
+
+extern "C" wind_status wind_kv_swap_out(const wind_kv_pool* dev, const int32_t* dev_bt,
+                                        wind_kv_pool* host, const int32_t* host_bt, int32_t n,
+                                        void* stream) {
+  if (!dev || !host) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
+  if (dev->desc.loc != WIND_LOC_DEVICE || host->desc.loc != WIND_LOC_HOST)
+    return fail(WIND_ERR_INVALID_ARG, "swap_out needs a device source and a host destination");
+  return wind_kv_migrate(dev, dev_bt, host, host_bt, n, dev->desc.first_layer,
+                         dev->desc.first_layer + dev->desc.n_layers, stream);
+}
+
+extern "C" wind_status wind_kv_swap_in(const wind_kv_pool* host, const int32_t* host_bt,
+                                       wind_kv_pool* dev, const int32_t* dev_bt, int32_t n,
+                                       void* stream) {
+  if (!dev || !host) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
+  if (dev->desc.loc != WIND_LOC_DEVICE || host->desc.loc != WIND_LOC_HOST)
+    return fail(WIND_ERR_INVALID_ARG, "swap_in needs a host source and a device destination");
+  return wind_kv_migrate(host, host_bt, dev, dev_bt, n, dev->desc.first_layer,
+                         dev->desc.first_layer + dev->desc.n_layers, stream);
+}
+
+extern "C" wind_status wind_kv_compact(wind_kv_pool* pool, const int32_t* src_bt,
+                                       const int32_t* dst_bt, int32_t n, void* stream) {
+  if (!pool) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
+  return wind_kv_migrate(pool, src_bt, pool, dst_bt, n, pool->desc.first_layer,
+                         pool->desc.first_layer + pool->desc.n_layers, stream);
+}
+
+// ------------------------------------------------------------------- layer flags
+
+extern "C" wind_status wind_kv_layer_ticket(const wind_kv_pool* dst, uint32_t* ticket) {
+  if (!dst || !ticket) return fail(WIND_ERR_INVALID_ARG, "NULL argument");
+  *ticket = dst->enqueued.load();
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_layer_wait(const wind_kv_pool* dst, int32_t layer, uint32_t ticket,
+                                          void* consumer) {
+  if (!dst) return fail(WIND_ERR_INVALID_ARG, "dst is NULL");
+  if (layer < dst->desc.first_layer || layer >= dst->desc.first_layer + dst->desc.n_layers)
+    return fail(WIND_ERR_LAYER_RANGE, "layer %d not in pool", layer);
+  static PFN_waitValue32 fn = driver_fn<PFN_waitValue32>("cuStreamWaitValue32");
+  if (!fn) return fail(WIND_ERR_CUDA, "cuStreamWaitValue32 entry point unavailable");
+  const uint32_t* f = dst->flags + (layer - dst->desc.first_layer);
+  CUresult r = fn(static_cast<CUstream>(consumer), reinterpret_cast<CUdeviceptr>(f), ticket,
+                  CU_STREAM_WAIT_VALUE_GEQ);
+  if (r != CUDA_SUCCESS) return fail(WIND_ERR_CUDA, "cuStreamWaitValue32 failed (CUresult %d)", static_cast<int>(r));
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_layer_count(const wind_kv_pool* dst, int32_t layer, uint32_t* value) {
+  if (!dst || !value) return fail(WIND_ERR_INVALID_ARG, "NULL argument");
+  if (layer < dst->desc.first_layer || layer >= dst->desc.first_layer + dst->desc.n_layers)
+    return fail(WIND_ERR_LAYER_RANGE, "layer %d not in pool", layer);
+  const uint32_t* f = dst->flags + (layer - dst->desc.first_layer);
+  if (dst->desc.loc == WIND_LOC_HOST) {
+    *value = *reinterpret_cast<const volatile uint32_t*>(f);
+    return WIND_OK;
+  }
+  DeviceGuard g(dst->desc.device);
+  WKV_CUDA(cudaMemcpy(value, f, sizeof(uint32_t), cudaMemcpyDeviceToHost), "cudaMemcpy(flag)");
+  return WIND_OK;
+}
+
+// ------------------------------------------------------------------- host logic
+
+extern "C" wind_status wind_kv_validate(const wind_kv_pool* src, const int32_t* sbt,
+                                        const wind_kv_pool* dst, const int32_t* dbt, int32_t n,
+                                        int32_t lo, int32_t hi) {
+  wind_status st = check_args(src, dst, n, lo, hi);
+  if (st != WIND_OK) return st;
+  if (n > 0 && (!sbt || !dbt)) return fail(WIND_ERR_INVALID_ARG, "block table is NULL");
+  return check_tables_host(src, sbt, dst, dbt, n);
+}
+
+extern "C" wind_status wind_kv_plan_compact(const uint8_t* live, int32_t n_slots, int32_t* src_bt,
+                                            int32_t* dst_bt, int32_t* n_moves) {
+  if (!n_moves || n_slots < 0 || (n_slots > 0 && !live)) return fail(WIND_ERR_INVALID_ARG, "bad arguments");
+  int32_t n_live = 0;
+  for (int32_t b = 0; b < n_slots; ++b) n_live += live[b] != 0;
+  // two fingers: `h` walks holes below n_live upward, `m` walks live slots at/above it upward
+  int32_t k = 0, h = 0, m = n_live;
+  for (;;) {
+    while (h < n_live && live[h]) ++h;
+    while (m < n_slots && !live[m]) ++m;
+    if (h >= n_live || m >= n_slots) break;
+    if (src_bt) src_bt[k] = m;
+    if (dst_bt) dst_bt[k] = h;
+    ++k, ++h, ++m;
+  }
+  *n_moves = k;
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_plan_rebalance(int32_t G, int32_t R, const int32_t* req_gpu,
+                                              const int32_t* req_blocks, int32_t* out_gpu,
+                                              int32_t* n_moves) {
+  if (G < 1 || R < 0 || !n_moves || (R > 0 && (!req_gpu || !req_blocks || !out_gpu)))
+    return fail(WIND_ERR_INVALID_ARG, "bad arguments");
+  std::vector<int64_t> load(G, 0);
+  // per GPU: candidate requests sorted by (blocks desc, id asc); removed lazily
+  std::vector<std::vector<int32_t>> by_gpu(G);
+  int64_t total = 0;
+  for (int32_t r = 0; r < R; ++r) {
+    if (req_gpu[r] < 0 || req_gpu[r] >= G || req_blocks[r] < 0)
+      return fail(WIND_ERR_INVALID_ARG, "request %d: bad gpu or block count", r);
+    out_gpu[r] = req_gpu[r];
+    load[req_gpu[r]] += req_blocks[r];
+    total += req_blocks[r];
+    if (req_blocks[r] > 0) by_gpu[req_gpu[r]].push_back(r);
+  }
+  for (auto& v : by_gpu)
+    std::sort(v.begin(), v.end(), [&](int32_t a, int32_t b) {
+      return req_blocks[a] != req_blocks[b] ? req_blocks[a] > req_blocks[b] : a < b;
+    });
+  const int64_t target = (total + G - 1) / G;
+  int32_t moves = 0;
+  for (;;) {
+    const int src = static_cast<int>(std::max_element(load.begin(), load.end()) - load.begin());
+    const int dst = static_cast<int>(std::min_element(load.begin(), load.end()) - load.begin());
+    if (load[src] <= target || src == dst) break;
+    const int64_t room = target - load[dst];
+    auto& v = by_gpu[src];
+    // first (longest, lowest id) request with blocks <= room: v is sorted by blocks desc
+    auto itr = std::lower_bound(v.begin(), v.end(), room, [&](int32_t r, int64_t rm) {
+      return req_blocks[r] > rm;
+    });
+    if (itr == v.end()) break;
+    const int32_t r = *itr;
+    v.erase(itr);
+    out_gpu[r] = dst;
+    load[src] -= req_blocks[r];
+    load[dst] += req_blocks[r];
+    ++moves;
+    // r never moves again: dst stays <= target, so it never becomes the source
+  }
+  *n_moves = moves;
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_check_device_error(const wind_kv_pool* p) {
+  if (!p) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
+  int32_t worst = 0;
+  for (int d = 0; d < kMaxDevices; ++d) {
+    DevCtx& c = g_dev[d];
+    if (!c.ready) continue;
+    if (p->desc.loc == WIND_LOC_DEVICE && d != p->desc.device) continue;
+    DeviceGuard g(d);
+    WKV_CUDA(cudaDeviceSynchronize(), "cudaDeviceSynchronize");
+    int32_t v = 0;
+    WKV_CUDA(cudaMemcpy(&v, c.err, sizeof v, cudaMemcpyDeviceToHost), "cudaMemcpy(err)");
+    WKV_CUDA(cudaMemset(c.err, 0, sizeof v), "cudaMemset(err)");
+    worst = std::max(worst, v);
+  }
+  if (worst == 0) return WIND_OK;
+  const char* what = worst == 4 ? "BLOCK_RANGE" : worst == 3 ? "DUP_DST" : "ALIAS";
+  return fail(WIND_ERR_DEVICE_CHECK, "device table check recorded %s", what);
+}
+
+// -------------------------------------------------------------------- tuning/misc
+
+extern "C" wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t) {
+  if (path < 0 || path > 2 || !t) return fail(WIND_ERR_INVALID_ARG, "bad path or NULL tuning");
+  std::lock_guard<std::mutex> lk(g_tune_mu);
+  wind_kv_tuning n = g_tune[path];
+  if (t->kernel < 0 || t->kernel > 2) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0, 1 or 2");
+  n.kernel = t->kernel;
+  if (t->ctas_per_sm) n.ctas_per_sm = t->ctas_per_sm;
+  if (t->stage_bytes) n.stage_bytes = t->stage_bytes;
+  if (t->stages) n.stages = t->stages;
+  n.max_ctas = t->max_ctas;
+  n.evict_first = t->evict_first;
+  if (n.ctas_per_sm < 1 || n.ctas_per_sm > 32) return fail(WIND_ERR_INVALID_ARG, "ctas_per_sm out of [1, 32]");
+  if (n.stage_bytes < 16 || n.stage_bytes % 16) return fail(WIND_ERR_INVALID_ARG, "stage_bytes must be a positive multiple of 16");
+  if (n.stages < 3 || n.stages > 16) return fail(WIND_ERR_INVALID_ARG, "stages out of [3, 16]");
+  if (tma_smem_bytes(n.stages, n.stage_bytes) > 227 * 1024)
+    return fail(WIND_ERR_INVALID_ARG, "stages * stage_bytes exceeds shared memory");
+  g_tune[path] = n;
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_get_tuning(int32_t path, wind_kv_tuning* t) {
+  if (path < 0 || path > 2 || !t) return fail(WIND_ERR_INVALID_ARG, "bad path or NULL tuning");
+  std::lock_guard<std::mutex> lk(g_tune_mu);
+  *t = g_tune[path];
+  return WIND_OK;
+}
+
+extern "C" uint64_t wind_kv_launch_count(void) { return g_launches.load(); }
+
+extern "C" const char* wind_kv_status_string(wind_status s) {
+  switch (s) {
+    case WIND_OK: return "WIND_OK";
+    case WIND_ERR_INVALID_ARG: return "WIND_ERR_INVALID_ARG";
+    case WIND_ERR_GEOMETRY: return "WIND_ERR_GEOMETRY";
+    case WIND_ERR_LAYER_RANGE: return "WIND_ERR_LAYER_RANGE";
+    case WIND_ERR_BLOCK_RANGE: return "WIND_ERR_BLOCK_RANGE";
+    case WIND_ERR_DUP_DST: return "WIND_ERR_DUP_DST";
+    case WIND_ERR_ALIAS: return "WIND_ERR_ALIAS";
+    case WIND_ERR_NO_PEER: return "WIND_ERR_NO_PEER";
+    case WIND_ERR_CUDA: return "WIND_ERR_CUDA";
+    case WIND_ERR_OOM: return "WIND_ERR_OOM";
+    case WIND_ERR_UNSUPPORTED: return "WIND_ERR_UNSUPPORTED";
+    case WIND_ERR_DEVICE_CHECK: return "WIND_ERR_DEVICE_CHECK";
+    default: return "WIND_ERR_UNKNOWN";
+  }
+}
+
+extern "C" const char* wind_kv_last_error(void) { return g_last_error.c_str(); }
+
+extern "C" const char* wind_kv_version(void) { return "wind_kv 0.1.0 (sm_100a)"; }

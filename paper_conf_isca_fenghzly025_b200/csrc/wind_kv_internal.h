@@ -1,0 +1,66 @@
+// wind_kv_internal.h — internal structures shared by the host side (wind_kv.cpp) and the
+// kernels (wind_kv_kernels.cu).  Not part of the ABI.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+
+#include "../../include/wind_kv.h"
+
+namespace wkv {
+
+// Ring of per-op, per-layer CTA-arrival counters on each executing device (A5).  An op
+// takes slot (seq % kCounterSlots); the last CTA to arrive on a layer resets the counter,
+// so a slot is reusable as soon as the op that used it has finished.
+constexpr int kCounterSlots = 64;
+constexpr int kMaxSegs = 32;  // segments (runs) per work unit = one warp's table window
+
+// One destination of a (possibly batched) migrate launch.
+struct Item {
+  const int32_t* sbt;
+  const int32_t* dbt;
+  uint8_t* dst_plane0;     // dst chunk (layer lo, K, block 0)
+  int64_t d_plane_stride;  // NB_dst * C
+  uint32_t* flags;         // dst layer_done[0 .. d_layers)
+  int32_t d_flag_lo;       // index of global layer lo in flags
+  int32_t d_layers;        // dst n_layers (for the out-of-range increments)
+  int32_t n;               // table entries
+  int32_t units;           // work units per (layer, kv) plane for this item
+  int32_t unit_base;       // prefix of `units` over previous items
+  int32_t host_flags;      // flags live in mapped host memory: bump by plain RMW, not red.sys
+};
+
+struct Params {
+  const uint8_t* src_plane0;  // src chunk (layer lo, K, block 0)
+  int64_t s_plane_stride;     // NB_src * C
+  int64_t chunk;              // C
+  int64_t units_per_plane;    // sum of items' units
+  int64_t total_units;        // planes * units_per_plane
+  uint32_t* counters;         // this op's counter slot, [hi - lo]
+  const int32_t* abort_word;  // debug pools: skip the copy if the device check fired
+  int32_t layer_lo, n_layers; // global lo, hi - lo
+  int32_t group;              // table entries per unit (>= 1; > 1 only when C < unit)
+  int32_t parts;              // units per chunk (> 1 only when C > unit)
+  int32_t part_bytes;         // bytes of a part (multiple of 16)
+  int32_t n_items;
+  int32_t evict_first;
+  int32_t stages;             // TMA ring depth
+  int32_t stage_bytes;        // TMA stage size
+  Item items[WIND_KV_MAX_BATCH];
+};
+
+enum Kernel { kAuto = 0, kTma = 1, kSimt = 2 };
+
+// Launchers (wind_kv_kernels.cu).  Return cudaGetLastError() after the launch.
+cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s);
+size_t tma_smem_bytes(int stages, int stage_bytes);
+cudaError_t prepare_kernels(int device, size_t max_tma_smem);
+
+// Debug-pool device table check (wind_kv_kernels.cu): records error codes in *err.
+cudaError_t launch_table_check(const int32_t* sbt, const int32_t* dbt, int32_t n,
+                               int32_t nb_src, int32_t nb_dst, int same_pool,
+                               uint32_t* scratch /* 2*max(nb) */, int32_t nb_scratch,
+                               int32_t* err, cudaStream_t s);
+
+}  // namespace wkv

@@ -1,0 +1,479 @@
+// wind_kv_kernels.cu — the sm_100a kernels of the paged KV-migration hot path.
+//
+// What they compute (include/wind_kv.h): for each (global layer
+// l in [lo, hi), kv in {K, V}) "plane" and each table entry i,
+//     dst[l][kv][dst_bt[i]] := src[l][kv][src_bt[i]]          (C contiguous bytes)
+// with the pools laid out [L][2][NB][H][bs][d] (reading R2), so every (layer, kv, block)
+// chunk is one contiguous C-byte span on both sides.  Pure data movement: no tensor
+// cores, no arithmetic on the payload (R13).
+//
+// Work decomposition (shared by both kernels).  A *unit* is at most `unit` bytes:
+//   C >= unit : one chunk split into `parts` pieces of part_bytes;
+//   C <  unit : a window of `group` (<= 32) consecutive table entries.  One warp loads
+//               the window, marks run heads where NOT (s_i = s_{i-1}+1 AND
+//               d_i = d_{i-1}+1) with __ballot_sync, and gives each run its segment
+//               index by prefix popcount (K3 run coalescer): a run of k
+//               adjacent blocks becomes ONE k*C-byte copy on both sides.
+// Units are numbered plane-major (layer ascending) and dealt to CTAs grid-stride,
+// so all CTAs sweep the layers together and a layer completes early (A5 streaming).
+//
+// Layer completion (A5).  When a CTA leaves layer l (its next unit is in a later layer, or
+// it is done) it makes its stores complete and system-visible, then adds 1 to this op's
+// arrival counter for l; the CTA that brings the counter to gridDim.x publishes
+// dst.layer_done[l] += 1 with a .release.sys reduction (a peer store over NVLink when dst
+// is remote) and resets the counter for the next op using the slot.
+//
+// Kernels.
+//   tma_copy_kernel  (K2): 2 warps per CTA.  Warp 0 = producer: decodes units and issues
+//     cp.async.bulk global->shared loads into an S-stage ring (mbarrier complete_tx).
+//     Warp 1 lane 0 = consumer: issues cp.async.bulk shared->global stores (bulk_group)
+//     and frees a stage once the store issued two units later has read it.  One thread
+//     keeps ~S*unit bytes in flight per CTA with a handful of instructions.
+//   simt_copy_kernel (K1): 512 threads per CTA, 16-byte ld.global.nc.L1::no_allocate /
+//     st.global vectors, 4 loads in flight per thread before the stores.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "wind_kv_internal.h"
+
+namespace wkv {
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+constexpr int kRelLag = 2;  // consumer frees stage of unit it-kRelLag (needs stages > 2)
+
+struct Seg {
+  const uint8_t* src;
+  uint8_t* dst;
+  uint32_t len;   // bytes (multiple of 16)
+  uint32_t soff;  // offset inside the unit's staging buffer
+};
+
+struct __align__(16) Desc {
+  int32_t nseg;   // -1 = end of work
+  int32_t plane;  // (l - lo) * 2 + kv
+  Seg segs[kMaxSegs];
+};
+
+// ----------------------------------------------------------------------- PTX helpers
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ uint64_t evict_first_policy() {
+  uint64_t pol;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+  return pol;
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+               "r"(bytes)
+               : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "WKV_WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      "@!p bra WKV_WAIT_%=;\n"
+      "}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+__device__ __forceinline__ void bulk_load(void* sdst, const void* gsrc, uint32_t bytes,
+                                          uint64_t* bar, bool ef, uint64_t pol) {
+  if (ef)
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1], %2, [%3], %4;" ::"r"(smem_u32(sdst)),
+        "l"(gsrc), "r"(bytes), "r"(smem_u32(bar)), "l"(pol)
+        : "memory");
+  else
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1], %2, [%3];" ::"r"(smem_u32(sdst)),
+        "l"(gsrc), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+__device__ __forceinline__ void bulk_store(void* gdst, const void* ssrc, uint32_t bytes,
+                                           bool ef, uint64_t pol) {
+  if (ef)
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group.L2::cache_hint [%0], [%1], %2, %3;"
+                 ::"l"(gdst), "r"(smem_u32(ssrc)), "r"(bytes), "l"(pol)
+                 : "memory");
+  else
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(gdst),
+                 "r"(smem_u32(ssrc)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;"); }
+
+template <int N>
+__device__ __forceinline__ void bulk_wait_read() {
+  asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
+
+__device__ __forceinline__ void bulk_wait_all() {
+  asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+
+__device__ __forceinline__ void fence_sys() {
+  asm volatile("fence.acq_rel.sys;" ::: "memory");
+}
+
+__device__ __forceinline__ void fence_async_global() {
+  asm volatile("fence.proxy.async.global;" ::: "memory");
+}
+
+__device__ __forceinline__ void red_release_sys_add(uint32_t* p, uint32_t v) {
+  asm volatile("red.release.sys.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+__device__ __forceinline__ int4 ld_stream(const int4* p) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p));
+  return r;
+}
+
+__device__ __forceinline__ int4 ld_stream_ef(const int4* p, uint64_t pol) {
+  int4 r;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.s32 {%0, %1, %2, %3}, [%4], %5;"
+               : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+               : "l"(p), "l"(pol));
+  return r;
+}
+
+__device__ __forceinline__ void st_stream(int4* p, const int4& v) {
+  asm volatile("st.global.L1::no_allocate.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(v.x),
+               "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+}
+
+__device__ __forceinline__ void st_stream_ef(int4* p, const int4& v, uint64_t pol) {
+  asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.s32 [%0], {%1, %2, %3, %4}, %5;"
+               ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w), "l"(pol)
+               : "memory");
+}
+
+// --------------------------------------------------------------------- work decoding
+
+// Decodes unit u into segments (called by a FULL warp; writes segs[] from the lanes that
+// own a segment).  Returns the (warp-uniform) segment count; *plane_out, *bytes_out.
+__device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs,
+                                           int32_t* plane_out, uint32_t* bytes_out) {
+  const int lane = threadIdx.x & 31;
+  const int64_t plane = u / p.units_per_plane;
+  int32_t r = static_cast<int32_t>(u - plane * p.units_per_plane);
+  int j = 0;
+  while (j + 1 < p.n_items && r >= p.items[j + 1].unit_base) ++j;
+  const Item& it = p.items[j];
+  r -= it.unit_base;
+  const uint8_t* splane = p.src_plane0 + plane * p.s_plane_stride;
+  uint8_t* dplane = it.dst_plane0 + plane * it.d_plane_stride;
+  const int64_t C = p.chunk;
+  *plane_out = static_cast<int32_t>(plane);
+  if (p.parts > 1) {  // one chunk, piece `part`
+    const int32_t i = r / p.parts;
+    const int32_t part = r - i * p.parts;
+    const int64_t off = static_cast<int64_t>(part) * p.part_bytes;
+    const int64_t rest = C - off;
+    const uint32_t len = static_cast<uint32_t>(rest < p.part_bytes ? rest : p.part_bytes);
+    if (lane == 0) {
+      const int32_t s = it.sbt[i], d = it.dbt[i];
+      segs[0].src = splane + s * C + off;
+      segs[0].dst = dplane + d * C + off;
+      segs[0].len = len;
+      segs[0].soff = 0;
+    }
+    *bytes_out = len;
+    return 1;
+  }
+  // a window of `group` entries: warp-ballot run coalescing (K3)
+  const int32_t i0 = r * p.group;
+  const int cnt = min(p.group, it.n - i0);
+  int32_t s = 0, d = 0;
+  if (lane < cnt) {
+    s = it.sbt[i0 + lane];
+    d = it.dbt[i0 + lane];
+  }
+  const int32_t ps = __shfl_up_sync(kFull, s, 1);
+  const int32_t pd = __shfl_up_sync(kFull, d, 1);
+  const bool head = lane < cnt && (lane == 0 || !(s == ps + 1 && d == pd + 1));
+  const uint32_t heads = __ballot_sync(kFull, head);
+  if (head) {
+    const int k = __popc(heads & ((1u << lane) - 1u));       // prefix popcount
+    const uint32_t later = heads & ~((2u << lane) - 1u);     // heads after this lane
+    const int end = later ? __ffs(later) - 1 : cnt;
+    segs[k].src = splane + s * C;
+    segs[k].dst = dplane + d * C;
+    segs[k].len = static_cast<uint32_t>((end - lane) * C);
+    segs[k].soff = static_cast<uint32_t>(lane * C);
+  }
+  *bytes_out = static_cast<uint32_t>(cnt * C);
+  return __popc(heads);
+}
+
+// Adds 1 to a layer flag with release semantics at system scope.  Device-memory flags
+// (local or peer) use a red.release.sys reduction; flags of a host pool (mapped pinned
+// memory, where PCIe may not carry atomics) use a volatile RMW + release store — the
+// executing device is then the only writer (wind_kv.h: one op at a time per host pool).
+__device__ __forceinline__ void bump_flag(uint32_t* f, bool host) {
+  if (!host) {
+    red_release_sys_add(f, 1u);
+  } else {
+    const uint32_t v = *reinterpret_cast<volatile uint32_t*>(f);
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(v + 1u) : "memory");
+  }
+}
+
+// Out-of-range layer flags: every op bumps every dst layer flag exactly once; the layers
+// it does not move are bumped at the start (see wind_kv.h, wind_kv_migrate).
+__device__ void publish_untouched_layers(const Params& p) {
+  for (int j = 0; j < p.n_items; ++j) {
+    const Item& it = p.items[j];
+    for (int f = 0; f < it.d_layers; ++f)
+      if (f < it.d_flag_lo || f >= it.d_flag_lo + p.n_layers) bump_flag(it.flags + f, it.host_flags);
+  }
+}
+
+// Arrive on layers [from, to) (global ids) of this op; the last CTA publishes.  Caller has
+// made this CTA's stores of those layers complete and ordered before this call.
+__device__ void arrive_layers(const Params& p, int32_t from, int32_t to) {
+  if (from >= to) return;
+  fence_sys();
+  for (int32_t l = from; l < to; ++l) {
+    uint32_t* c = p.counters + (l - p.layer_lo);
+    const uint32_t old = atomicAdd(c, 1u);
+    if (old == gridDim.x - 1) {
+      fence_sys();
+      for (int j = 0; j < p.n_items; ++j)
+        bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (l - p.layer_lo), p.items[j].host_flags);
+      *reinterpret_cast<volatile uint32_t*>(c) = 0u;  // slot reusable by a later op
+    }
+  }
+}
+
+// ------------------------------------------------------------------- K2: TMA staged
+
+__global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__ Params p) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  const int S = p.stages;
+  const uint32_t SB = static_cast<uint32_t>(p.stage_bytes);
+  uint8_t* buf = smem;
+  Desc* desc = reinterpret_cast<Desc*>(smem + static_cast<size_t>(S) * SB);
+  uint64_t* full = reinterpret_cast<uint64_t*>(desc + S);
+  uint64_t* empty = full + S;
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const bool ef = p.evict_first != 0;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    if (blockIdx.x == 0) publish_untouched_layers(p);
+  }
+  __syncthreads();
+
+  if (warp == 0) {  // ------------------------------------------------ producer warp
+    const uint64_t pol = ef ? evict_first_policy() : 0;
+    const int64_t total = (p.abort_word && *p.abort_word) ? 0 : p.total_units;
+    int it = 0;
+    for (int64_t u = blockIdx.x;; u += gridDim.x, ++it) {
+      const int st = it % S;
+      if (it >= S) mbar_wait(&empty[st], ((it / S) & 1) ^ 1);
+      if (u >= total) {
+        if (lane == 0) {
+          desc[st].nseg = -1;
+          mbar_arrive(&full[st]);
+        }
+        break;
+      }
+      int32_t plane;
+      uint32_t bytes;
+      const int nseg = decode_unit(p, u, desc[st].segs, &plane, &bytes);
+      __syncwarp();
+      if (lane == 0) {
+        desc[st].nseg = nseg;
+        desc[st].plane = plane;
+        mbar_arrive_expect_tx(&full[st], bytes);
+        uint8_t* sbuf = buf + static_cast<size_t>(st) * SB;
+        for (int k = 0; k < nseg; ++k) {
+          const Seg& g = desc[st].segs[k];
+          bulk_load(sbuf + g.soff, g.src, g.len, &full[st], ef, pol);
+        }
+      }
+      __syncwarp();
+    }
+  } else if (lane == 0) {  // ---------------------------------------- consumer thread
+    const uint64_t pol = ef ? evict_first_policy() : 0;
+    int32_t cur = p.layer_lo;  // layers < cur have been arrived on by this CTA
+    for (int it = 0;; ++it) {
+      const int st = it % S;
+      mbar_wait(&full[st], (it / S) & 1);
+      const int nseg = desc[st].nseg;
+      if (nseg < 0) break;
+      const int32_t layer = p.layer_lo + desc[st].plane / 2;
+      if (layer > cur) {  // this CTA is done with layers [cur, layer)
+        bulk_wait_all();
+        fence_async_global();
+        arrive_layers(p, cur, layer);
+        cur = layer;
+      }
+      const uint8_t* sbuf = buf + static_cast<size_t>(st) * SB;
+      for (int k = 0; k < nseg; ++k) {
+        const Seg& g = desc[st].segs[k];
+        bulk_store(g.dst, sbuf + g.soff, g.len, ef, pol);
+      }
+      bulk_commit();
+      bulk_wait_read<kRelLag>();  // stores of units <= it - kRelLag have read their stage
+      if (it >= kRelLag) mbar_arrive(&empty[(it - kRelLag) % S]);
+    }
+    bulk_wait_all();
+    fence_async_global();
+    arrive_layers(p, cur, p.layer_lo + p.n_layers);
+  }
+}
+
+// ------------------------------------------------------------------ K1: SIMT vectors
+
+constexpr int kSimtThreads = 512;
+constexpr int kSimtUnroll = 4;
+
+__global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_constant__ Params p) {
+  __shared__ Seg segs[kMaxSegs];
+  __shared__ int32_t s_nseg, s_plane;
+  const int tid = threadIdx.x;
+  const bool ef = p.evict_first != 0;
+  const uint64_t pol = ef ? evict_first_policy() : 0;
+  if (blockIdx.x == 0 && tid == 0) publish_untouched_layers(p);
+  int32_t cur = p.layer_lo;
+  const int64_t total = (p.abort_word && *p.abort_word) ? 0 : p.total_units;
+  for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
+    if (tid < 32) {
+      int32_t plane;
+      uint32_t bytes;
+      const int n = decode_unit(p, u, segs, &plane, &bytes);
+      if (tid == 0) {
+        s_nseg = n;
+        s_plane = plane;
+      }
+    }
+    __syncthreads();
+    const int32_t layer = p.layer_lo + s_plane / 2;
+    if (layer > cur) {  // uniform: every thread of the CTA left layers [cur, layer)
+      if (tid == 0) arrive_layers(p, cur, layer);
+      cur = layer;
+    }
+    const int nseg = s_nseg;
+    for (int k = 0; k < nseg; ++k) {
+      const int4* s = reinterpret_cast<const int4*>(segs[k].src);
+      int4* d = reinterpret_cast<int4*>(segs[k].dst);
+      const int nv = static_cast<int>(segs[k].len >> 4);
+      for (int v = tid; v < nv; v += kSimtUnroll * kSimtThreads) {
+        int4 r[kSimtUnroll];
+#pragma unroll
+        for (int q = 0; q < kSimtUnroll; ++q) {
+          const int vi = v + q * kSimtThreads;
+          if (vi < nv) r[q] = ef ? ld_stream_ef(s + vi, pol) : ld_stream(s + vi);
+        }
+#pragma unroll
+        for (int q = 0; q < kSimtUnroll; ++q) {
+          const int vi = v + q * kSimtThreads;
+          if (vi < nv) {
+            if (ef)
+              st_stream_ef(d + vi, r[q], pol);
+            else
+              st_stream(d + vi, r[q]);
+          }
+        }
+      }
+    }
+    __syncthreads();  // all stores of this unit issued; segs may be overwritten
+  }
+  if (tid == 0) arrive_layers(p, cur, p.layer_lo + p.n_layers);
+}
+
+// -------------------------------------------------------- debug-pool device table check
+
+__global__ void table_count_kernel(const int32_t* sbt, const int32_t* dbt, int32_t n,
+                                   int32_t nb_src, int32_t nb_dst, uint32_t* dcnt,
+                                   uint32_t* scnt, int32_t* err) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t s = sbt[i], d = dbt[i];
+    if (s < 0 || s >= nb_src || d < 0 || d >= nb_dst) {
+      atomicMax(reinterpret_cast<int*>(err), 4);  // 4 = BLOCK_RANGE (rank of precedence)
+      continue;
+    }
+    atomicAdd(dcnt + d, 1u);
+    atomicAdd(scnt + s, 1u);
+  }
+}
+
+__global__ void table_judge_kernel(const int32_t* sbt, const int32_t* dbt, int32_t n,
+                                   int32_t nb_src, int32_t nb_dst, int same_pool,
+                                   const uint32_t* dcnt, const uint32_t* scnt, int32_t* err) {
+  for (int32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += gridDim.x * blockDim.x) {
+    const int32_t s = sbt[i], d = dbt[i];
+    if (s < 0 || s >= nb_src || d < 0 || d >= nb_dst) continue;
+    if (dcnt[d] > 1) atomicMax(reinterpret_cast<int*>(err), 3);  // DUP_DST
+    if (same_pool && scnt[d] > (s == d ? 1u : 0u)) atomicMax(reinterpret_cast<int*>(err), 2);  // ALIAS
+  }
+}
+
+}  // namespace
+
+size_t tma_smem_bytes(int stages, int stage_bytes) {
+  return static_cast<size_t>(stages) * stage_bytes + static_cast<size_t>(stages) * sizeof(Desc) +
+         2 * static_cast<size_t>(stages) * sizeof(uint64_t);
+}
+
+cudaError_t prepare_kernels(int device, size_t max_tma_smem) {
+  (void)device;
+  return cudaFuncSetAttribute(tma_copy_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              static_cast<int>(max_tma_smem));
+}
+
+cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s) {
+  if (kernel == kTma) {
+    tma_copy_kernel<<<grid, 64, tma_smem_bytes(p.stages, p.stage_bytes), s>>>(p);
+  } else {
+    simt_copy_kernel<<<grid, kSimtThreads, 0, s>>>(p);
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_table_check(const int32_t* sbt, const int32_t* dbt, int32_t n,
+                               int32_t nb_src, int32_t nb_dst, int same_pool,
+                               uint32_t* scratch, int32_t nb_scratch, int32_t* err,
+                               cudaStream_t s) {
+  uint32_t* dcnt = scratch;
+  uint32_t* scnt = scratch + nb_scratch;
+  cudaError_t e = cudaMemsetAsync(scratch, 0, sizeof(uint32_t) * 2 * nb_scratch, s);
+  if (e != cudaSuccess) return e;
+  const int grid = n / 256 + 1 < 1024 ? n / 256 + 1 : 1024;
+  table_count_kernel<<<grid, 256, 0, s>>>(sbt, dbt, n, nb_src, nb_dst, dcnt, scnt, err);
+  table_judge_kernel<<<grid, 256, 0, s>>>(sbt, dbt, n, nb_src, nb_dst, same_pool, dcnt, scnt, err);
+  return cudaGetLastError();
+}
+
+}  // namespace wkv
