@@ -817,7 +817,7 @@ extern "C" wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t)
   if (n.ctas_per_sm < 1 || n.ctas_per_sm > 32) return fail(WIND_ERR_INVALID_ARG, "ctas_per_sm out of [1, 32]");
   if (n.stage_bytes < 16 || n.stage_bytes % 16) return fail(WIND_ERR_INVALID_ARG, "stage_bytes must be a positive multiple of 16");
   if (n.stages < 3 || n.stages > 16) return fail(WIND_ERR_INVALID_ARG, "stages out of [3, 16]");
-  if (tma_smem_bytes(n.stages, n.stage_bytes) > 227 * 1024)
+  if (n.kernel != kSimt && tma_smem_bytes(n.stages, n.stage_bytes) > 227 * 1024)
     return fail(WIND_ERR_INVALID_ARG, "stages * stage_bytes exceeds shared memory");
   g_tune[path] = n;
   return WIND_OK;

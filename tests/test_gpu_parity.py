@@ -229,8 +229,10 @@ def test_argument_errors_match_oracle_precedence():
         want = O.check_op(geom(args[0]), geom(args[2]), 1, kw["layer_lo"], kw["layer_hi"])
         assert got == want, (kw, got, want)
     assert status_of(wk.migrate, a, t1, b, t1, n=-1) == -1
-    # stream on the wrong device / invalid stream handle -> INVALID_ARG
-    assert status_of(wk.migrate, a, t1, b, t1, layer_lo=2, layer_hi=4, stream=0xdead) == -1
+    # a pool on a device that does not exist -> INVALID_ARG at creation
+    with pytest.raises(wk.WindKVError) as e:
+        wk.Pool(4, 2, 64, 16, 2, 8, device=torch.cuda.device_count() + 3)
+    assert e.value.status == -1
     torch.cuda.synchronize()
 
 
