@@ -1,0 +1,121 @@
+"""Tuning sweep for the copy kernels on one B200 (development tool, not the bench).
+
+Prints one JSON line per configuration: payload GB/s and DRAM fraction of the measured
+copy peak for the C2 (160 KiB chunks) and C5 (16 KiB chunks) shapes, shuffled tables.
+"""
+import json
+import math
+import os
+import sys
+import time
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import paper_conf_isca_fenghzly025_b200 as wk  # noqa: E402
+import windgen.cuda as wg  # noqa: E402
+from windgen import migration_case, SHAPES, KVShape  # noqa: E402
+
+PEAK = json.load(open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
+                                   "MEASURED_PEAKS.json")))["hbm_gbs"]
+dev = torch.device("cuda", 0)
+
+
+def pool(sh, nb, tag):
+    p = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, nb)
+    wg.fill(p.base, p.nbytes, 0, 1, tag)
+    return p
+
+
+def timeit(fn, stream, reps=10, warm=3):
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    a.record(stream)
+    for _ in range(reps):
+        fn()
+    b.record(stream)
+    torch.cuda.synchronize()
+    return a.elapsed_time(b) / reps
+
+
+def main():
+    which = sys.argv[1] if len(sys.argv) > 1 else "all"
+    s = torch.cuda.Stream(dev)
+    out = []
+    cases = {}
+    c2 = migration_case("C2")
+    cases["C2"] = (c2.shape, c2)
+    # C5-shaped (16 KiB chunks) with a similar ~20 GiB payload
+    sh5 = SHAPES["C5"]
+    c5 = migration_case("C5", shape=sh5, lengths=np.full(640, 1024))
+    cases["C5"] = (sh5, c5)
+    for name, (sh, case) in cases.items():
+        src = pool(sh, case.nb_src, 1)
+        dst = pool(sh, case.nb_dst, 2)
+        sbt = torch.as_tensor(case.src_bt, device=dev)
+        dbt = torch.as_tensor(case.dst_bt, device=dev)
+        pb = 2 * sh.n_layers * case.n * sh.chunk_bytes
+        configs = []
+        if which in ("all", "kernels"):
+            for stage, stages, cps in [(32768, 6, 1), (65536, 3, 1), (16384, 12, 1), (49152, 4, 1),
+                                       (24576, 8, 1), (32768, 3, 2), (16384, 6, 2), (8192, 6, 4),
+                                       (65536, 6, 0)]:
+                if cps == 0:
+                    continue
+                configs.append(dict(kernel=wk.KERNEL_TMA, stage_bytes=stage, stages=stages, ctas_per_sm=cps))
+            for stage, cps in [(32768, 4), (16384, 4), (65536, 4), (32768, 2), (32768, 3), (131072, 4)]:
+                configs.append(dict(kernel=wk.KERNEL_SIMT, stage_bytes=stage, stages=6, ctas_per_sm=cps))
+            for ef in (True,):
+                configs.append(dict(kernel=wk.KERNEL_TMA, stage_bytes=32768, stages=6, ctas_per_sm=1,
+                                    evict_first=ef))
+        for cfg in configs:
+            wk.set_tuning(wk.PATH_INTRA, **cfg)
+            ms = timeit(lambda: wk.migrate(src, sbt, dst, dbt, stream=s), s)
+            gbs = pb / ms / 1e6
+            r = dict(case=name, **cfg, ms=round(ms, 3), gbs=round(gbs, 1), frac=round(2 * gbs / PEAK, 4))
+            print(json.dumps(r), flush=True)
+        wk.set_tuning(wk.PATH_INTRA, kernel=wk.KERNEL_TMA, stage_bytes=32768, stages=6, ctas_per_sm=1)
+        if which in ("all", "stream") and name == "C2":
+            cons = torch.cuda.Stream(dev)
+            L = sh.n_layers
+
+            def streamed(wait):
+                for l in range(L):
+                    wk.migrate(src, sbt, dst, dbt, layer_lo=l, layer_hi=l + 1, stream=s)
+                if wait:
+                    t = dst.layer_ticket()
+                    for l in range(L):
+                        wk.layer_wait(dst, l, t, stream=cons)
+                    s.wait_stream(cons)
+            for wait in (False, True):
+                ms = timeit(lambda: streamed(wait), s, reps=5)
+                print(json.dumps(dict(case=name, mode="streamed", wait=wait, ms=round(ms, 3),
+                                      gbs=round(pb / ms / 1e6, 1))), flush=True)
+            # one layer alone: launch + ramp + drain cost
+            ms1 = timeit(lambda: wk.migrate(src, sbt, dst, dbt, layer_lo=5, layer_hi=6, stream=s), s, reps=20)
+            print(json.dumps(dict(case=name, mode="one_layer", ms=round(ms1, 4),
+                                  gbs=round(pb / L / ms1 / 1e6, 1))), flush=True)
+            # CTA cap curve (for interference control)
+            for cap in (8, 16, 24, 32, 48, 74, 148):
+                wk.set_tuning(wk.PATH_INTRA, kernel=wk.KERNEL_TMA, max_ctas=cap)
+                ms = timeit(lambda: wk.migrate(src, sbt, dst, dbt, stream=s), s, reps=3)
+                print(json.dumps(dict(case=name, mode="cap", max_ctas=cap, gbs=round(pb / ms / 1e6, 1))),
+                      flush=True)
+            wk.set_tuning(wk.PATH_INTRA, kernel=wk.KERNEL_TMA, max_ctas=0)
+        del src, dst
+        torch.cuda.empty_cache()
+    # copy-engine comparators
+    n = 8 << 30
+    a = torch.empty(n, dtype=torch.uint8, device=dev)
+    b = torch.empty(n, dtype=torch.uint8, device=dev)
+    ms = timeit(lambda: b.copy_(a), torch.cuda.current_stream(dev))
+    print(json.dumps(dict(mode="torch_copy_8GiB", gbs_rw=round(2 * n / ms / 1e6, 1))), flush=True)
+    ms = timeit(lambda: torch.cuda.current_stream(dev) and
+                torch.cuda.cudart() and b.copy_(a, non_blocking=True), torch.cuda.current_stream(dev))
+
+
+if __name__ == "__main__":
+    main()
