@@ -286,7 +286,172 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
     ms_ce = time_device(lambda: hbuf.copy_(dbuf, non_blocking=True), steps, warmup,
                         torch.cuda.current_stream(device)) / steps
     out["c1_swap"]["copy_engine_d2h_gbs"] = round(pb / ms_ce / 1e6, 2)
-    del dpool, dpool2, hpool
+    del dpool, dpool2, hpool, hbuf, dbuf
+    torch.cuda.empty_cache()
+
+    # (5) interference with a co-running decode stream (C3)
+    out["c3_interference"] = run_interference(wk, device, peaks)
+    return out
+
+
+def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:
+    """S§8(d) interference, C3 (OPT-66B KV, 64 layers x 72 heads x d 128, fp16): the victim
+    is paged decode attention over 16 x 2048 resident tokens (the Fig. 8 decode set,
+    P:251) = 72 GiB of KV read per step (64 layer launches) on a HIGH-priority stream; the
+    migration moves 4 x 2048-token long-context requests (P:227, 18 GiB) on a LOW-priority
+    side stream, looped to cover every victim step.  On one GPU the migration is
+    intra-device (reads AND writes this HBM); a CTA cap emulates the source-side HBM load
+    of an NVLink push (8 CTAs ~ 365 GB/s payload = 730 GB/s of DRAM traffic, about what a
+    770 GB/s peer push reads on its source GPU)."""
+    import torch
+    import victim
+    from windgen import migration_case, SHAPES
+    sh = SHAPES["C3"]
+    dev = torch.device("cuda", device)
+    B, ctx_len, bs = 16, 2048, sh.block_size
+    nbv = B * ctx_len // bs
+    vpool = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, bs, sh.elem_bytes, nbv, device=device)
+    vt = vpool.tensor().view(torch.float16)
+    g = torch.Generator(device=dev).manual_seed(0)
+    step_elems = 1 << 28
+    for o in range(0, vt.numel(), step_elems):
+        n = min(step_elems, vt.numel() - o)
+        vt[o:o + n].normal_(generator=g)
+    perm = torch.randperm(nbv, generator=torch.Generator().manual_seed(1)).to(torch.int32)
+    bt = perm.view(B, ctx_len // bs).to(dev)
+    ctx = torch.full((B,), ctx_len, dtype=torch.int32, device=dev)
+    q = torch.randn(B, sh.n_kv_heads, sh.head_dim, device=dev, dtype=torch.float16)
+    bps = 32
+    scratch = torch.empty(victim.scratch_floats(B, sh.n_kv_heads, ctx_len // bs, bps), device=dev)
+    out = torch.empty(B, sh.n_kv_heads, sh.head_dim, device=dev)
+    plane = nbv * sh.chunk_bytes
+    hi_s = torch.cuda.Stream(device, priority=-1)
+    lo_s = torch.cuda.Stream(device, priority=0)
+
+    def victim_step():
+        for l in range(sh.n_layers):
+            kp = vpool.base + (2 * l) * plane
+            victim.decode_attention(q, kp, kp + plane, bt, ctx, sh.n_kv_heads, bs, scratch, out,
+                                    blocks_per_split=bps, stream=hi_s.cuda_stream)
+
+    def victim_run(n):
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
+        ev[0].record(hi_s)
+        for i in range(n):
+            victim_step()
+            ev[i + 1].record(hi_s)
+        return ev
+
+    for _ in range(5):
+        victim_step()
+    torch.cuda.synchronize()
+    ev = victim_run(n_victim_steps)
+    torch.cuda.synchronize()
+    alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]
+    t_alone = float(np.median(alone))
+    kv_read = B * ctx_len * sh.n_layers * 2 * sh.n_kv_heads * sh.head_dim * sh.elem_bytes
+    res = {"victim_ms_alone": round(t_alone, 3),
+           "victim_hbm_frac": round(kv_read / t_alone / 1e6 / peaks["hbm_gbs"], 3),
+           "victim": "paged decode attention, 16 x 2048 tok, 64 layers, 72 heads (C3)"}
+
+    case = migration_case("C3")
+    src = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
+    dst = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag)
+    sbt = torch.as_tensor(case.src_bt, device=dev)
+    dbt = torch.as_tensor(case.dst_bt, device=dev)
+    pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
+    saved = wk.get_tuning(wk.PATH_INTRA)
+    for cap in (8, 16, 0):
+        wk.set_tuning(wk.PATH_INTRA, **{**saved, "max_ctas": cap})
+        t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, stream=lo_s), 2, 3, lo_s) / 2
+        k = int(math.ceil(n_victim_steps * t_alone * 3.0 / t_mig)) + 2
+        m0, m1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        m0.record(lo_s)
+        for _ in range(k):
+            wk.migrate(src, sbt, dst, dbt, stream=lo_s)
+        m1.record(lo_s)
+        ev = victim_run(n_victim_steps)
+        torch.cuda.synchronize()
+        with_mig = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]
+        covered = ev[n_victim_steps].elapsed_time(m1) > 0  # migration outlived the victim
+        t_with = float(np.median(with_mig))
+        res[f"cap{cap or 'none'}"] = {
+            "migration_gbs_alone": round(pb / t_mig / 1e6, 1),
+            "victim_ms_with_migration": round(t_with, 3),
+            "slowdown": round(t_with / t_alone - 1.0, 4),
+            "migration_covered_all_victim_steps": bool(covered)}
+    wk.set_tuning(wk.PATH_INTRA, **saved)
+    del vpool, src, dst
+    return res
+
+
+def run_all_to_all(wk, rank, world, device, peaks, steps=5, warmup=3) -> dict:
+    """A8 at N > 1: C5 (Llama-3-8B GQA fp8, 1024 long-tail requests) placed with skewed
+    weights over the ranks; every rank derives the same plan (uniform hash shuffle =
+    bandwidth headline; greedy rebalance = realistic), imports every peer's pool and pushes
+    its outgoing blocks to all peers in one wind_kv_migrate_batch launch."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_isca_fenghzly025_b200 import parallel, rebalance
+    from windgen import (SHAPES, request_lengths, skewed_placement, blocks_for_tokens,
+                         hash_shuffle_dest)
+    sh = SHAPES["C5"]
+    lens = request_lengths("C5")
+    gpu = skewed_placement(lens.size, world, 4005)
+    blocks = blocks_for_tokens(lens, 16).astype(np.int32)
+    loads = np.bincount(gpu, weights=blocks, minlength=world).astype(np.int64)
+    nb = int(loads.max() + math.ceil(1.5 * blocks.sum() / world))
+    rng = [np.random.default_rng(5000 + g) for g in range(world)]
+    perms = [r.permutation(nb) for r in rng]
+    pos = [0] * world
+    tables = []
+    for r in range(lens.size):
+        g = int(gpu[r])
+        tables.append(perms[g][pos[g]:pos[g] + blocks[r]].astype(np.int32))
+        pos[g] += int(blocks[r])
+    free = []
+    for g in range(world):
+        m = np.ones(nb, bool)
+        m[perms[g][:pos[g]]] = False
+        free.append(m)
+    dev = torch.device("cuda", device)
+    pool = make_pool(wk, sh, nb, device, 3005, 10 + rank)
+    handles = parallel.exchange_handles(pool.export())
+    peers = {g: wk.Pool.import_(h, device) for g, h in enumerate(handles) if g != rank}
+    s = torch.cuda.Stream(device)
+    keep = []
+
+    def to_dev(a):
+        t = torch.as_tensor(a, device=dev)
+        keep.append(t)
+        return t
+    out = {}
+    for kind in ("shuffle", "rebalance"):
+        if kind == "shuffle":
+            plan = rebalance.plan_exchange(world, gpu, tables, free,
+                                           hash_shuffle_dest(lens.size, world, 4005))
+        else:
+            plan = rebalance.plan_rebalance_exchange(world, gpu, tables, free)
+        items = plan.items_for(rank)
+        batch = [(peers[d], to_dev(sb), to_dev(db)) for d, sb, db in items]
+        sent = sum(int(sb.size) for _, sb, _ in items)
+
+        def step():
+            for k in range(0, len(batch), wk.MAX_BATCH):
+                wk.migrate_batch(pool, batch[k:k + wk.MAX_BATCH], 0, sh.n_layers, stream=s)
+        if not batch:
+            step = lambda: None  # noqa: E731
+        ms = time_device(step, steps, warmup, s, barrier=dist.barrier) / steps
+        ms_max, = parallel.max_over_ranks([ms])
+        tot = plan.blocks_moved * 2 * sh.n_layers * sh.chunk_bytes
+        per_gpu_egress = sent * 2 * sh.n_layers * sh.chunk_bytes / ms / 1e6
+        out[kind] = {"aggregate_gbs": round(tot / ms_max / 1e6, 1), "ms": round(ms_max, 3),
+                     "blocks_moved": int(plan.blocks_moved),
+                     "rank0_egress_gbs": round(per_gpu_egress, 1) if rank == 0 else None,
+                     "nvlink_frac_per_gpu": round(tot / world / ms_max / 1e6 / 900.0, 4)}
+    for p in peers.values():
+        p.destroy()
     return out
 
 
@@ -310,24 +475,19 @@ def run_gpu(args) -> None:
     barrier = (lambda: dist.barrier()) if world > 1 else None
     peaks = load_peaks()
 
+    from paper_conf_isca_fenghzly025_b200 import parallel
     case = migration_case(args.config, variant=args.variant)
     sh = case.shape
-    role = "solo"
-    if world > 1:
-        if rank % 2 == 0 and rank + 1 < world:
-            role = "push"
-        elif rank % 2 == 1:
-            role = "decode"
+    role, partner = parallel.pair_role(rank, world)
     src = dst = None
     if role in ("solo", "push"):
         src = make_pool(wk, sh, case.nb_src, local, case.content_seed, case.src_tag)
     if role in ("solo", "decode"):
         dst = make_pool(wk, sh, case.nb_dst, local, case.content_seed, case.dst_tag)
     if world > 1:
-        handles = [None] * world
-        dist.all_gather_object(handles, dst.export() if role == "decode" else None)
+        handles = parallel.exchange_handles(dst.export() if role == "decode" else None)
         if role == "push":
-            dst = wk.Pool.import_(handles[rank + 1], local)
+            dst = wk.Pool.import_(handles[partner], local)
     stream = torch.cuda.Stream(local)
     sbt = torch.as_tensor(case.src_bt, device=dev)
     dbt = torch.as_tensor(case.dst_bt, device=dev)
@@ -364,15 +524,14 @@ def run_gpu(args) -> None:
 
     ms_e2e_local = time_device(e2e_step, max(3, args.steps // 2), 2, stream, barrier) / max(3, args.steps // 2)
 
-    # max over ranks
-    t = torch.tensor([ms_step_local, ms_e2e_local], dtype=torch.float64)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-    ms_step, ms_e2e = float(t[0]), float(t[1])
-    n_movers = sum(1 for r in range(world) if not (r % 2 == 1) or world == 1) if world > 1 else 1
-    if world > 1:
-        n_movers = world // 2 + (world % 2)
+    ms_step, ms_e2e = parallel.max_over_ranks([ms_step_local, ms_e2e_local])
+    n_movers = parallel.movers(world)
     total_bytes = pb * n_movers
+    a2a = None
+    if world > 1 and args.scenarios:
+        del src, dst
+        torch.cuda.empty_cache()
+        a2a = run_all_to_all(wk, rank, world, local, peaks)
     value = total_bytes / ms_step / 1e6  # GB/s
     e2e_value = total_bytes / ms_e2e / 1e6
 
@@ -391,7 +550,9 @@ def run_gpu(args) -> None:
                     "frac": round(kernel_gbs / 900.0, 4), "traffic": None, "peak_src": "nominal",
                     "per_launch_bytes": pb}
         extra["roofline"] = roof
-        extra["parity"] = parity_sample(wk, case, src, dst, lo, hi) if role == "solo" else None
+        extra["parity"] = parity_sample(wk, case, src, dst, lo, hi) if world == 1 else None
+        if a2a is not None:
+            extra["scenarios"] = {"c5_all_to_all": a2a}
         if world == 1 and not args.no_cpu_baseline:
             extra["cpu_baseline"] = cpu_baseline(case)
         if world == 1 and args.scenarios:

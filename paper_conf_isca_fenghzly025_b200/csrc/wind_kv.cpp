@@ -126,9 +126,9 @@ wind_status dev_ctx(int dev, DevCtx** out) {
 
 std::mutex g_tune_mu;
 wind_kv_tuning g_tune[3] = {
-    /* INTRA */ {kTma, 1, 32768, 6, 0, 0},
-    /* PEER  */ {kSimt, 4, 32768, 6, 0, 0},
-    /* HOST  */ {kSimt, 4, 32768, 6, 0, 0},
+    /* INTRA */ {kTma, 1, 49152, 4, 0, 0, 2},  // sweep r01: 0.998 (C2) / 0.985 (C5) of HBM copy
+    /* PEER  */ {kSimt, 4, 32768, 6, 0, 0, 0},
+    /* HOST  */ {kSimt, 4, 32768, 6, 0, 0, 0},
 };
 
 }  // namespace
@@ -576,6 +576,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   p.src_plane0 = src->base + static_cast<int64_t>(lo - src->desc.first_layer) * 2 * src->desc.n_blocks * C;
   p.s_plane_stride = static_cast<int64_t>(src->desc.n_blocks) * C;
   p.evict_first = t.evict_first;
+  p.store_lag = t.store_lag;
   p.stages = t.stages;
   p.stage_bytes = t.stage_bytes;
   int32_t base_units = 0;
@@ -814,6 +815,8 @@ extern "C" wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t)
   if (t->stages) n.stages = t->stages;
   n.max_ctas = t->max_ctas;
   n.evict_first = t->evict_first;
+  n.store_lag = t->store_lag;
+  if (n.store_lag < 0 || n.store_lag >= n.stages) return fail(WIND_ERR_INVALID_ARG, "store_lag out of [0, stages)");
   if (n.ctas_per_sm < 1 || n.ctas_per_sm > 32) return fail(WIND_ERR_INVALID_ARG, "ctas_per_sm out of [1, 32]");
   if (n.stage_bytes < 16 || n.stage_bytes % 16) return fail(WIND_ERR_INVALID_ARG, "stage_bytes must be a positive multiple of 16");
   if (n.stages < 3 || n.stages > 16) return fail(WIND_ERR_INVALID_ARG, "stages out of [3, 16]");

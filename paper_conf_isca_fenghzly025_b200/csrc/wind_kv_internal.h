@@ -45,6 +45,7 @@ struct Params {
   int32_t part_bytes;         // bytes of a part (multiple of 16)
   int32_t n_items;
   int32_t evict_first;
+  int32_t store_lag;          // TMA consumer: units whose stores may still read smem
   int32_t stages;             // TMA ring depth
   int32_t stage_bytes;        // TMA stage size
   Item items[WIND_KV_MAX_BATCH];

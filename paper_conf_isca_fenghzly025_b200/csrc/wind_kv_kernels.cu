@@ -40,7 +40,6 @@ namespace wkv {
 namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
-constexpr int kRelLag = 2;  // consumer frees stage of unit it-kRelLag (needs stages > 2)
 
 struct Seg {
   const uint8_t* src;
@@ -244,12 +243,36 @@ __device__ __forceinline__ void bump_flag(uint32_t* f, bool host) {
 }
 
 // Out-of-range layer flags: every op bumps every dst layer flag exactly once; the layers
-// it does not move are bumped at the start (see wind_kv.h, wind_kv_migrate).
+// it does not move are bumped at the start (see wind_kv.h, wind_kv_migrate).  No data is
+// published with them, so the bumps are relaxed (a release per flag costs a system-scope
+// fence each, ~1 us); the caller is a thread off the copy's critical path.
 __device__ void publish_untouched_layers(const Params& p) {
   for (int j = 0; j < p.n_items; ++j) {
     const Item& it = p.items[j];
-    for (int f = 0; f < it.d_layers; ++f)
-      if (f < it.d_flag_lo || f >= it.d_flag_lo + p.n_layers) bump_flag(it.flags + f, it.host_flags);
+    for (int f = 0; f < it.d_layers; ++f) {
+      if (f >= it.d_flag_lo && f < it.d_flag_lo + p.n_layers) continue;
+      uint32_t* fl = it.flags + f;
+      if (!it.host_flags) {
+        asm volatile("red.relaxed.sys.global.add.u32 [%0], 1;" ::"l"(fl) : "memory");
+      } else {
+        const uint32_t v = *reinterpret_cast<volatile uint32_t*>(fl);
+        *reinterpret_cast<volatile uint32_t*>(fl) = v + 1u;
+      }
+    }
+  }
+}
+
+// cp.async.bulk.wait_group.read needs an immediate: dispatch the runtime lag.
+__device__ __forceinline__ void bulk_wait_read_n(int n) {
+  switch (n) {
+    case 0: bulk_wait_read<0>(); break;
+    case 1: bulk_wait_read<1>(); break;
+    case 2: bulk_wait_read<2>(); break;
+    case 3: bulk_wait_read<3>(); break;
+    case 4: bulk_wait_read<4>(); break;
+    case 5: bulk_wait_read<5>(); break;
+    case 6: bulk_wait_read<6>(); break;
+    default: bulk_wait_read<7>(); break;
   }
 }
 
@@ -290,9 +313,9 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
       mbar_init(&empty[i], 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    if (blockIdx.x == 0) publish_untouched_layers(p);
   }
   __syncthreads();
+  if (blockIdx.x == 0 && threadIdx.x == 33) publish_untouched_layers(p);  // an idle consumer lane
 
   if (warp == 0) {  // ------------------------------------------------ producer warp
     const uint64_t pol = ef ? evict_first_policy() : 0;
@@ -326,6 +349,9 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
     }
   } else if (lane == 0) {  // ---------------------------------------- consumer thread
     const uint64_t pol = ef ? evict_first_policy() : 0;
+    // stores allowed to be still reading their stage: half the ring (the other half is
+    // the producer's load lookahead)
+    const int lag = p.store_lag > 0 ? p.store_lag : (S / 2 > 0 ? S / 2 : 1);
     int32_t cur = p.layer_lo;  // layers < cur have been arrived on by this CTA
     for (int it = 0;; ++it) {
       const int st = it % S;
@@ -345,8 +371,8 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
         bulk_store(g.dst, sbuf + g.soff, g.len, ef, pol);
       }
       bulk_commit();
-      bulk_wait_read<kRelLag>();  // stores of units <= it - kRelLag have read their stage
-      if (it >= kRelLag) mbar_arrive(&empty[(it - kRelLag) % S]);
+      bulk_wait_read_n(lag);  // stores of units <= it - lag have read their stage
+      if (it >= lag) mbar_arrive(&empty[(it - lag) % S]);
     }
     bulk_wait_all();
     fence_async_global();
@@ -365,7 +391,7 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
   const int tid = threadIdx.x;
   const bool ef = p.evict_first != 0;
   const uint64_t pol = ef ? evict_first_policy() : 0;
-  if (blockIdx.x == 0 && tid == 0) publish_untouched_layers(p);
+  if (blockIdx.x == 0 && tid == 32) publish_untouched_layers(p);  // not the decoding warp
   int32_t cur = p.layer_lo;
   const int64_t total = (p.abort_word && *p.abort_word) ? 0 : p.total_units;
   for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {

@@ -60,13 +60,13 @@ def main():
         pb = 2 * sh.n_layers * case.n * sh.chunk_bytes
         configs = []
         if which in ("all", "kernels"):
-            for stage, stages, cps in [(32768, 6, 1), (65536, 3, 1), (16384, 12, 1), (49152, 4, 1),
-                                       (24576, 8, 1), (32768, 3, 2), (16384, 6, 2), (8192, 6, 4),
-                                       (65536, 6, 0)]:
-                if cps == 0:
-                    continue
-                configs.append(dict(kernel=wk.KERNEL_TMA, stage_bytes=stage, stages=stages, ctas_per_sm=cps))
-            for stage, cps in [(32768, 4), (16384, 4), (65536, 4), (32768, 2), (32768, 3), (131072, 4)]:
+            for stage, stages, cps, lag in [(32768, 6, 1, 3), (32768, 6, 1, 2), (32768, 6, 1, 4),
+                                            (49152, 4, 1, 2), (49152, 4, 1, 1), (65536, 3, 1, 1),
+                                            (40960, 5, 1, 2), (24576, 8, 1, 4), (16384, 12, 1, 6),
+                                            (16384, 6, 2, 3), (32768, 3, 2, 1), (8192, 6, 4, 3)]:
+                configs.append(dict(kernel=wk.KERNEL_TMA, stage_bytes=stage, stages=stages,
+                                    ctas_per_sm=cps, store_lag=lag))
+            for stage, cps in [(32768, 4), (65536, 2), (131072, 4)]:
                 configs.append(dict(kernel=wk.KERNEL_SIMT, stage_bytes=stage, stages=6, ctas_per_sm=cps))
             for ef in (True,):
                 configs.append(dict(kernel=wk.KERNEL_TMA, stage_bytes=32768, stages=6, ctas_per_sm=1,
