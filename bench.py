@@ -291,7 +291,57 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
 
     # (5) interference with a co-running decode stream (C3)
     out["c3_interference"] = run_interference(wk, device, peaks)
+    torch.cuda.empty_cache()
+
+    # (6) stall-free rescheduling of P:120's request (NEXT-1)
+    out["stall_free"] = run_stall_free(wk, device)
     return out
+
+
+def run_stall_free(wk, device, cap_ctas: int = 16) -> dict:
+    """NEXT-1: one OPT-13B request of 2048 tokens (1.5625 GiB of KV) keeps
+    decoding while it migrates; it is blocked only for the final stage.  The migration is
+    capped at `cap_ctas` CTAs (~700 GB/s, an NVLink-rate push) and compared with a
+    stop-the-world migration of the same request at the same rate."""
+    import torch
+    from paper_conf_isca_fenghzly025_b200 import stall_free
+    from windgen import SHAPES
+    import windgen.cuda as wg
+    sh = SHAPES["C2"]
+    bs, T0, nb, capb = sh.block_size, 2048, 600, 300
+    dev = torch.device("cuda", device)
+    rng = np.random.default_rng(0)
+    ss = rng.permutation(nb)[:capb].astype(np.int32)
+    ds = rng.permutation(nb)[:capb].astype(np.int32)
+    src = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, bs, sh.elem_bytes, nb, device=device)
+    dst = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, bs, sh.elem_bytes, nb, device=device)
+    wg.fill(src.base, src.nbytes, 0, 1, 1)
+    saved = wk.get_tuning(wk.PATH_INTRA)
+    wk.set_tuning(wk.PATH_INTRA, **{**saved, "max_ctas": cap_ctas})
+    mig, dec = torch.cuda.Stream(device), torch.cuda.Stream(device)
+    st, dt = torch.as_tensor(ss, device=dev), torch.as_tensor(ds, device=dev)
+    step = stall_free.append_token_kernel_factory(src, ss, dec)
+    step(T0)
+    torch.cuda.synchronize()
+    # decode-step time of the synthetic append and the stop-the-world migration time
+    t0 = time.perf_counter()
+    for t in range(T0, T0 + 20):
+        step(t)
+        dec.synchronize()
+    step_ms = (time.perf_counter() - t0) / 20 * 1e3
+    n0 = T0 // bs
+    stw = time_device(lambda: wk.migrate(src, st, dst, dt, n=n0, stream=mig), 3, 2, mig) / 3
+    bw = n0 * 2 * sh.n_layers * sh.chunk_bytes / stw / 1e6
+    theta = stall_free.default_theta(max(step_ms, 0.05), bw, sh.n_layers, sh.chunk_bytes)
+    res = stall_free.migrate_stall_free(src, st, dst, dt, T0, theta, step, mig, dec)
+    wk.set_tuning(wk.PATH_INTRA, **saved)
+    del src, dst
+    return {"request": "OPT-13B, 2048 tokens at start (P:120)", "cap_ctas": cap_ctas,
+            "migration_gbs": round(bw, 1), "stop_the_world_ms": round(stw, 3),
+            "theta_blocks": theta, "stages": len(res.stages), "tokens_decoded_while_migrating":
+            int(sum(res.appends)), "pause_ms": round(res.pause_ms, 3),
+            "blocked_time_reduction": round(1 - res.pause_ms / stw, 4),
+            "blocks_sent": res.blocks_sent}
 
 
 def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:

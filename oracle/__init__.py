@@ -89,6 +89,7 @@ def _lib():
             "or_plan_rebalance": (ct.c_int, [I32, I32, P, P, P, P]),
             "or_migrate_mt": (ct.c_int, [P, G, P, P, G, P, I32, I32, I32, I32]),
             "or_hw_threads": (I32, []),
+            "or_stall_free_plan": (ct.c_int, [I32, I32, I32, P, I32, P, P, P, P]),
         }
         for name, (res, args) in sig.items():
             f = getattr(lib, name)
@@ -196,6 +197,21 @@ def migrate_mt(src: np.ndarray, gs: Geom, src_bt, dst: np.ndarray, gd: Geom, dst
     s, d = _i32(src_bt), _i32(dst_bt)
     return int(_lib().or_migrate_mt(_p(src), ct.byref(gs.c()), _p(s), _p(dst),
                                     ct.byref(gd.c()), _p(d), s.size, lo, hi, n_threads))
+
+
+def stall_free_plan(T0: int, bs: int, theta: int, appends) -> tuple[list, int]:
+    """O8: [(begin_block, end_block), ...] (the last = pause stage) and the pause token
+    count, for per-stage append counts `appends` (len = max_stages)."""
+    a = _i32(appends)
+    m = a.size
+    b = np.zeros(m + 1, np.int32)
+    e = np.zeros(m + 1, np.int32)
+    ns = np.zeros(1, np.int32)
+    ft = np.zeros(1, np.int32)
+    rc = int(_lib().or_stall_free_plan(T0, bs, theta, _p(a), m, _p(b), _p(e), _p(ns), _p(ft)))
+    if rc != OK:
+        raise ValueError(f"stall_free_plan rc={rc}")
+    return [(int(b[k]), int(e[k])) for k in range(ns[0])], int(ft[0])
 
 
 def hw_threads() -> int:

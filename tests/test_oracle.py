@@ -343,3 +343,57 @@ def test_plan_rebalance_invariants():
                         and load[dst] + b <= target]
                 assert not fits
             assert moves == int((out != gpu).sum())
+
+
+# ------------------------------------------------------ O8 stall-free staging (NEXT-1)
+
+def closed_form_stall_free(T0, bs, theta, appends):
+    """Independent closed form of P:231's protocol (reading R6): with tok_k the tokens when
+    stage k starts (prefix sums of the appends), stage k sends [floor(tok_{k-1}/bs),
+    floor(tok_k/bs)); the pause comes after the first stage k with
+    ceil(tok_{k+1}/bs) - floor(tok_k/bs) <= theta (or the last allowed stage)."""
+    tok = T0 + np.concatenate([[0], np.cumsum(appends)])
+    m = len(appends)
+    fl = tok // bs
+    ce = -(-tok // bs)
+    stages = [(0, int(fl[0]))]
+    for k in range(m):
+        if ce[k + 1] - fl[k] <= theta or k + 1 == m:
+            stages.append((int(fl[k]), int(ce[k + 1])))
+            return stages, int(tok[k + 1])
+        stages.append((int(fl[k]), int(fl[k + 1])))
+    raise AssertionError
+
+
+def test_stall_free_plan_matches_closed_form():
+    rng = np.random.default_rng(0)
+    for trial in range(3000):
+        bs = int(rng.choice([1, 2, 16]))
+        T0 = int(rng.integers(0, 300))
+        theta = int(rng.integers(0, 6))
+        m = int(rng.integers(1, 12))
+        appends = rng.integers(0, 40, m)
+        got = O.stall_free_plan(T0, bs, theta, appends)
+        assert got == closed_form_stall_free(T0, bs, theta, appends), (T0, bs, theta, appends)
+
+
+def test_stall_free_plan_invariants():
+    """P9: every block of the request at the pause is sent exactly once, in order (so the
+    bytes sent are ceil(final/bs) * 2 * L * C); stages before the pause carry only full
+    blocks; the pause leaves at most theta blocks (unless max stages forced it)."""
+    rng = np.random.default_rng(1)
+    for trial in range(2000):
+        bs, T0, theta = 16, int(rng.integers(0, 5000)), int(rng.integers(1, 8))
+        appends = rng.integers(0, 64, 20)
+        stages, final = O.stall_free_plan(T0, bs, theta, appends)
+        cover = [b for s, e in stages for b in range(s, e)]
+        assert cover == list(range(-(-final // bs)))
+        tok = T0
+        for k, (s, e) in enumerate(stages[:-1]):
+            assert e <= tok // bs  # only blocks full when the stage starts
+            tok += int(appends[k])
+        s, e = stages[-1]
+        if len(stages) - 1 < len(appends):
+            assert e - s <= theta
+    # theta larger than any request: one bulk stage, then the pause sends the tail
+    assert O.stall_free_plan(100, 16, 10**6, [5, 5]) == ([(0, 6), (6, 7)], 105)
