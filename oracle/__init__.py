@@ -90,6 +90,8 @@ def _lib():
             "or_migrate_mt": (ct.c_int, [P, G, P, P, G, P, I32, I32, I32, I32]),
             "or_hw_threads": (I32, []),
             "or_stall_free_plan": (ct.c_int, [I32, I32, I32, P, I32, P, P, P, P]),
+            "or_check_op_heads": (ct.c_int, [G, G, I32, I32, I32, I32, I32, I32]),
+            "or_migrate_heads": (ct.c_int, [P, G, P, P, G, P, I32, I32, I32, I32, I32, I32]),
         }
         for name, (res, args) in sig.items():
             f = getattr(lib, name)
@@ -139,6 +141,19 @@ def migrate(src: np.ndarray, gs: Geom, src_bt, dst: np.ndarray, gd: Geom, dst_bt
     assert src.size == gs.pool_bytes and dst.size == gd.pool_bytes
     return int(_lib().or_migrate(_p(src), ct.byref(gs.c()), _p(s), _p(dst), ct.byref(gd.c()),
                                  _p(d), s.size, lo, hi))
+
+
+def check_op_heads(gs: Geom, gd: Geom, n, lo, hi, sh0, dh0, nh) -> int:
+    return int(_lib().or_check_op_heads(ct.byref(gs.c()), ct.byref(gd.c()), n, lo, hi, sh0, dh0, nh))
+
+
+def migrate_heads(src: np.ndarray, gs: Geom, src_bt, dst: np.ndarray, gd: Geom, dst_bt,
+                  lo: int, hi: int, src_head_lo: int, dst_head_lo: int, n_heads: int) -> int:
+    """NEXT-3 head-range migrate (TP reshard); `src is dst` = same pool."""
+    s, d = _i32(src_bt), _i32(dst_bt)
+    assert src.size == gs.pool_bytes and dst.size == gd.pool_bytes
+    return int(_lib().or_migrate_heads(_p(src), ct.byref(gs.c()), _p(s), _p(dst), ct.byref(gd.c()),
+                                       _p(d), s.size, lo, hi, src_head_lo, dst_head_lo, n_heads))
 
 
 def swap_out(dev: np.ndarray, gdev: Geom, dev_bt, host: np.ndarray, ghost: Geom, host_bt) -> int:

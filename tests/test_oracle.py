@@ -397,3 +397,64 @@ def test_stall_free_plan_invariants():
             assert e - s <= theta
     # theta larger than any request: one bulk stage, then the pause sends the tail
     assert O.stall_free_plan(100, 16, 10**6, [5, 5]) == ([(0, 6), (6, 7)], 105)
+
+
+# ------------------------------------------------------------ NEXT-3 head-range migrate
+
+def test_migrate_heads_brute_force():
+    """Element-wise: D[l, kv, dbt[i], dh0 + h] = S[l, kv, sbt[i], sh0 + h] via 7-D numpy
+    indexing, all other bytes unchanged; random geometries, offsets and tables."""
+    rng = np.random.default_rng(3)
+    for trial in range(200):
+        Hs, Hd = int(rng.integers(1, 5)), int(rng.integers(1, 5))
+        nh = int(rng.integers(1, min(Hs, Hd) + 1))
+        sh0, dh0 = int(rng.integers(0, Hs - nh + 1)), int(rng.integers(0, Hd - nh + 1))
+        gs = O.Geom(0, 2, Hs, 8, 2, 1, 5)
+        gd = O.Geom(0, 3, Hd, 8, 2, 1, 4)
+        n = int(rng.integers(0, 4))
+        sbt = rng.integers(0, 5, n).astype(np.int32)
+        dbt = rng.permutation(4)[:n].astype(np.int32)
+        lo, hi = 0, int(rng.integers(0, 3))
+        src, dst = rand_pool(gs, trial), rand_pool(gd, trial + 99)
+        want = dst.copy()
+        W = brute.as7d(want, gd)
+        S = brute.as7d(src, gs)
+        for i in range(n):
+            for l in range(lo, hi):
+                for kv in range(2):
+                    for h in range(nh):
+                        W[l, kv, dbt[i], dh0 + h] = S[l, kv, sbt[i], sh0 + h]
+        assert O.migrate_heads(src, gs, sbt, dst, gd, dbt, lo, hi, sh0, dh0, nh) == O.OK
+        np.testing.assert_array_equal(dst, want)
+
+
+def test_tp_reshard_equals_full_migrate():
+    """[TP-2 -> TP-1] (Fig. 3): two prefill ranks, each holding half the heads,
+    push their halves into one decode pool; the result equals migrating the unsharded
+    pool directly, and migrate_heads over all heads equals migrate."""
+    H = 8
+    full = O.Geom(0, 3, H, 16, 16, 2, 20)
+    half = O.Geom(0, 3, H // 2, 16, 16, 2, 20)
+    src = rand_pool(full, 1)
+    S = src.reshape(3, 2, 20, H, -1)
+    shards = [np.ascontiguousarray(S[:, :, :, r * H // 2:(r + 1) * H // 2]).reshape(-1) for r in range(2)]
+    sbt, dbt = np.array([3, 7, 19, 0], np.int32), np.array([5, 6, 1, 2], np.int32)
+    want = rand_pool(full, 2)
+    got = want.copy()
+    assert O.migrate(src, full, sbt, want, full, dbt, 0, 3) == O.OK
+    for r in range(2):
+        assert O.migrate_heads(shards[r], half, sbt, got, full, dbt, 0, 3, 0, r * H // 2, H // 2) == O.OK
+    np.testing.assert_array_equal(got, want)
+    got2 = rand_pool(full, 2)
+    assert O.migrate_heads(src, full, sbt, got2, full, dbt, 0, 3, 0, 0, H) == O.OK
+    np.testing.assert_array_equal(got2, want)
+
+
+def test_migrate_heads_errors():
+    gs, gd = O.Geom(0, 2, 4, 8, 2, 1, 5), O.Geom(0, 2, 2, 8, 2, 1, 5)
+    assert O.check_op_heads(gs, gd, 1, 0, 2, 0, 0, 2) == O.OK
+    assert O.check_op_heads(gs, gd, 1, 0, 2, 0, 1, 2) == O.GEOMETRY   # leaves dst heads
+    assert O.check_op_heads(gs, gd, 1, 0, 2, 3, 0, 2) == O.GEOMETRY   # leaves src heads
+    assert O.check_op_heads(gs, gd, 1, 0, 2, 0, 0, 0) == O.INVALID_ARG
+    assert O.check_op_heads(gs, O.Geom(0, 2, 2, 16, 2, 1, 5), 1, 0, 2, 0, 0, 1) == O.GEOMETRY
+    assert O.check_op_heads(gs, gd, 1, 0, 3, 0, 0, 1) == O.LAYER_RANGE
