@@ -170,6 +170,19 @@ wind_status wind_kv_swap_in(const wind_kv_pool* host, const int32_t* host_bt,
 wind_status wind_kv_compact(wind_kv_pool* pool, const int32_t* src_bt, const int32_t* dst_bt,
                             int32_t n_blocks, void* stream);
 
+/* Head-range migrate (NEXT-3, TP reshard): under tensor parallelism KV is sharded by head
+ * (Table 3: every placement is TP-2) and prefill / decode placements may differ
+ * ([TP-2, TP-1], Fig. 3).  For l in [lo, hi), kv, i, h in [0, n_heads):
+ *   dst[l][kv][dst_bt[i]][dst_head_lo + h] := src_before[l][kv][src_bt[i]][src_head_lo + h]
+ * (each head tile is bs*d*e_b contiguous bytes; H may differ between the pools).
+ * Errors: INVALID_ARG (n_heads < 1, negative offsets) > GEOMETRY (d / bs / e_b differ, or a
+ * head range leaves its pool) > LAYER_RANGE; UNSUPPORTED if bs*d*e_b % 16 != 0.  Same
+ * execution, table contract, tickets and flags as wind_kv_migrate. */
+wind_status wind_kv_migrate_heads(const wind_kv_pool* src, const int32_t* src_bt, wind_kv_pool* dst,
+                                  const int32_t* dst_bt, int32_t n_blocks, int32_t layer_lo,
+                                  int32_t layer_hi, int32_t src_head_lo, int32_t dst_head_lo,
+                                  int32_t n_heads, void* stream);
+
 /* One entry of a batched migrate: several (dst pool, tables) pairs from ONE source pool,
  * executed by one persistent launch (all-to-all rebalancing, A8: a GPU pushing to up to
  * 7 peers at once).  Each entry takes its own ticket on its dst. */

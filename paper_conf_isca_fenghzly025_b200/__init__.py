@@ -19,7 +19,7 @@ from typing import Optional, Sequence
 import numpy as np
 
 __all__ = [
-    "WindKVError", "Pool", "lib", "migrate", "migrate_batch", "swap_out", "swap_in", "compact",
+    "WindKVError", "Pool", "lib", "migrate", "migrate_batch", "migrate_heads", "swap_out", "swap_in", "compact",
     "layer_wait", "validate", "plan_compact", "plan_rebalance", "check_device_error",
     "set_tuning", "get_tuning", "launch_count", "STATUS", "PATH_INTRA", "PATH_PEER", "PATH_HOST",
     "KERNEL_AUTO", "KERNEL_TMA", "KERNEL_SIMT", "EXPORTED_SYMBOLS",
@@ -45,7 +45,8 @@ MAX_BATCH = 16
 EXPORTED_SYMBOLS = [
     "wind_kv_pool_create", "wind_kv_pool_destroy", "wind_kv_pool_info", "wind_kv_pool_flags",
     "wind_kv_pool_export", "wind_kv_pool_import", "wind_kv_migrate", "wind_kv_swap_out",
-    "wind_kv_swap_in", "wind_kv_compact", "wind_kv_migrate_batch", "wind_kv_layer_ticket",
+    "wind_kv_swap_in", "wind_kv_compact", "wind_kv_migrate_batch", "wind_kv_migrate_heads",
+    "wind_kv_layer_ticket",
     "wind_kv_layer_wait", "wind_kv_layer_count", "wind_kv_validate", "wind_kv_plan_compact",
     "wind_kv_plan_rebalance", "wind_kv_check_device_error", "wind_kv_set_tuning",
     "wind_kv_get_tuning", "wind_kv_launch_count", "wind_kv_status_string", "wind_kv_last_error",
@@ -106,6 +107,7 @@ def lib() -> ct.CDLL:
         "wind_kv_swap_in": [P, P, P, P, I32, P],
         "wind_kv_compact": [P, P, P, I32, P],
         "wind_kv_migrate_batch": [P, ct.POINTER(MigrateItem), I32, I32, I32, P],
+        "wind_kv_migrate_heads": [P, P, P, P, I32, I32, I32, I32, I32, I32, P],
         "wind_kv_layer_ticket": [P, ct.POINTER(U32)],
         "wind_kv_layer_wait": [P, I32, U32, P],
         "wind_kv_layer_count": [P, I32, ct.POINTER(U32)],
@@ -296,6 +298,19 @@ def migrate(src: Pool, src_bt, dst: Pool, dst_bt, n: Optional[int] = None,
     hi = min(src.layers[1], dst.layers[1]) if layer_hi is None else layer_hi
     _check(lib().wind_kv_migrate(src.handle, _ptr(src_bt), dst.handle, _ptr(dst_bt), n, lo, hi,
                                  _stream(stream, _exec_device(src, dst))))
+
+
+def migrate_heads(src: Pool, src_bt, dst: Pool, dst_bt, src_head_lo: int, dst_head_lo: int,
+                  n_heads: int, n: Optional[int] = None, layer_lo: Optional[int] = None,
+                  layer_hi: Optional[int] = None, stream=None) -> None:
+    """wind_kv_migrate_heads: heads [src_head_lo, +n_heads) of each source block into heads
+    [dst_head_lo, +n_heads) of the destination block (TP reshard, NEXT-3)."""
+    n = _len(src_bt) if n is None else n
+    lo = max(src.layers[0], dst.layers[0]) if layer_lo is None else layer_lo
+    hi = min(src.layers[1], dst.layers[1]) if layer_hi is None else layer_hi
+    _check(lib().wind_kv_migrate_heads(src.handle, _ptr(src_bt), dst.handle, _ptr(dst_bt), n, lo, hi,
+                                       src_head_lo, dst_head_lo, n_heads,
+                                       _stream(stream, _exec_device(src, dst))))
 
 
 def migrate_batch(src: Pool, items: Sequence[tuple], layer_lo: int, layer_hi: int,

@@ -435,13 +435,31 @@ wind_status check_tables_host(const wind_kv_pool* src, const int32_t* sbt,
   return WIND_OK;
 }
 
+// A head sub-range of every block (NEXT-3, TP reshard); n < 0 = whole chunks.
+struct HeadRange {
+  int32_t src_lo = 0, dst_lo = 0, n = -1;
+};
+
 // Argument checks shared by every op: INVALID_ARG > GEOMETRY > LAYER_RANGE.
 wind_status check_args(const wind_kv_pool* src, const wind_kv_pool* dst, int32_t n, int32_t lo,
-                       int32_t hi) {
+                       int32_t hi, const HeadRange& hr = HeadRange()) {
   if (!src || !dst) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
   if (n < 0) return fail(WIND_ERR_INVALID_ARG, "n_blocks < 0");
-  if (!same_geometry(src->desc, dst->desc))
-    return fail(WIND_ERR_GEOMETRY, "pools differ in H/d/block_size/elem_bytes");
+  if (hr.n < 0) {
+    if (!same_geometry(src->desc, dst->desc))
+      return fail(WIND_ERR_GEOMETRY, "pools differ in H/d/block_size/elem_bytes");
+  } else {
+    if (hr.n < 1 || hr.src_lo < 0 || hr.dst_lo < 0)
+      return fail(WIND_ERR_INVALID_ARG, "head range: n_heads >= 1 and offsets >= 0 required");
+    const wind_kv_pool_desc &a = src->desc, &b = dst->desc;
+    if (a.head_dim != b.head_dim || a.block_size != b.block_size || a.elem_bytes != b.elem_bytes)
+      return fail(WIND_ERR_GEOMETRY, "pools differ in d/block_size/elem_bytes");
+    if (hr.src_lo + hr.n > a.n_kv_heads || hr.dst_lo + hr.n > b.n_kv_heads)
+      return fail(WIND_ERR_GEOMETRY, "head range leaves a pool (src %d+%d of %d, dst %d+%d of %d)",
+                  hr.src_lo, hr.n, a.n_kv_heads, hr.dst_lo, hr.n, b.n_kv_heads);
+    if ((static_cast<int64_t>(a.block_size) * a.head_dim * a.elem_bytes) % 16 != 0)
+      return fail(WIND_ERR_UNSUPPORTED, "head tile bs*d*e_b must be a multiple of 16 bytes");
+  }
   if (lo > hi) return fail(WIND_ERR_LAYER_RANGE, "layer_lo %d > layer_hi %d", lo, hi);
   if (lo < hi && (!layers_inside(src->desc, lo, hi) || !layers_inside(dst->desc, lo, hi)))
     return fail(WIND_ERR_LAYER_RANGE, "layers [%d, %d) not inside both pools", lo, hi);
@@ -517,13 +535,13 @@ wind_status debug_check(DevCtx* ctx, int exec, const wind_kv_pool* src, const Op
 
 // The common op: src -> items[] over layers [lo, hi) on `stream`.
 wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
-                   int32_t hi, void* stream) {
+                   int32_t hi, void* stream, const HeadRange& hr = HeadRange()) {
   if (!src) return fail(WIND_ERR_INVALID_ARG, "src pool is NULL");
   if (n_items < 1 || n_items > WIND_KV_MAX_BATCH) return fail(WIND_ERR_INVALID_ARG, "n_items out of range");
   int exec = -1, path = 0;
   wind_status st;
   for (int j = 0; j < n_items; ++j) {
-    if ((st = check_args(src, items[j].dst, items[j].n, lo, hi)) != WIND_OK) return st;
+    if ((st = check_args(src, items[j].dst, items[j].n, lo, hi, hr)) != WIND_OK) return st;
     if (items[j].n > 0 && (!items[j].sbt || !items[j].dbt)) return fail(WIND_ERR_INVALID_ARG, "block table is NULL");
     for (int k = 0; k < j; ++k)
       if (items[k].dst == items[j].dst) return fail(WIND_ERR_INVALID_ARG, "batch destinations must be distinct");
@@ -559,22 +577,26 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
 
   Params p;
   memset(&p, 0, sizeof p);
-  const int64_t C = src->chunk;
+  const int64_t CS = src->chunk;
+  const int64_t tile = static_cast<int64_t>(src->desc.block_size) * src->desc.head_dim * src->desc.elem_bytes;
+  const int64_t CP = hr.n < 0 ? CS : hr.n * tile;  // bytes copied per (layer, kv, block)
   const int64_t unit = t.stage_bytes;
-  p.chunk = C;
-  if (C >= unit) {
-    p.parts = static_cast<int32_t>((C + unit - 1) / unit);
-    p.part_bytes = static_cast<int32_t>((((C + p.parts - 1) / p.parts) + 15) / 16 * 16);
+  p.s_chunk = CS;
+  p.copy = CP;
+  if (CP >= unit) {
+    p.parts = static_cast<int32_t>((CP + unit - 1) / unit);
+    p.part_bytes = static_cast<int32_t>((((CP + p.parts - 1) / p.parts) + 15) / 16 * 16);
     p.group = 1;
   } else {
     p.parts = 1;
-    p.part_bytes = static_cast<int32_t>(C);
-    p.group = static_cast<int32_t>(std::min<int64_t>(kMaxSegs, unit / C));
+    p.part_bytes = static_cast<int32_t>(CP);
+    p.group = static_cast<int32_t>(std::min<int64_t>(kMaxSegs, unit / CP));
   }
   p.layer_lo = lo;
   p.n_layers = hi - lo;
-  p.src_plane0 = src->base + static_cast<int64_t>(lo - src->desc.first_layer) * 2 * src->desc.n_blocks * C;
-  p.s_plane_stride = static_cast<int64_t>(src->desc.n_blocks) * C;
+  p.src_plane0 = src->base + static_cast<int64_t>(lo - src->desc.first_layer) * 2 * src->desc.n_blocks * CS +
+                 (hr.n < 0 ? 0 : hr.src_lo * tile);
+  p.s_plane_stride = static_cast<int64_t>(src->desc.n_blocks) * CS;
   p.evict_first = t.evict_first;
   p.store_lag = t.store_lag;
   p.stages = t.stages;
@@ -588,8 +610,12 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     q.sbt = it.sbt;
     q.dbt = it.dbt;
     q.n = it.n;
-    q.dst_plane0 = d->base + static_cast<int64_t>(lo - d->desc.first_layer) * 2 * d->desc.n_blocks * C;
-    q.d_plane_stride = static_cast<int64_t>(d->desc.n_blocks) * C;
+    const int64_t CD = d->chunk;
+    q.dst_plane0 = d->base + static_cast<int64_t>(lo - d->desc.first_layer) * 2 * d->desc.n_blocks * CD +
+                   (hr.n < 0 ? 0 : hr.dst_lo * tile);
+    q.d_plane_stride = static_cast<int64_t>(d->desc.n_blocks) * CD;
+    q.d_chunk = CD;
+    q.coalesce = (CP == CS && CP == CD) ? 1 : 0;
     q.flags = d->flags;
     q.d_flag_lo = lo - d->desc.first_layer;
     q.d_layers = d->desc.n_layers;
@@ -629,6 +655,19 @@ extern "C" wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* s
   if (!dst) return fail(WIND_ERR_INVALID_ARG, "dst pool is NULL");
   OpItem it{dst, src_bt, dst_bt, n_blocks};
   return run_op(src, &it, 1, layer_lo, layer_hi, stream);
+}
+
+extern "C" wind_status wind_kv_migrate_heads(const wind_kv_pool* src, const int32_t* src_bt,
+                                             wind_kv_pool* dst, const int32_t* dst_bt, int32_t n_blocks,
+                                             int32_t layer_lo, int32_t layer_hi, int32_t src_head_lo,
+                                             int32_t dst_head_lo, int32_t n_heads, void* stream) {
+  if (!dst) return fail(WIND_ERR_INVALID_ARG, "dst pool is NULL");
+  OpItem it{dst, src_bt, dst_bt, n_blocks};
+  HeadRange hr;
+  hr.src_lo = src_head_lo;
+  hr.dst_lo = dst_head_lo;
+  hr.n = n_heads < 0 ? 0 : n_heads;  // n_heads < 1 is rejected by check_args
+  return run_op(src, &it, 1, layer_lo, layer_hi, stream, hr);
 }
 
 extern "C" wind_status wind_kv_migrate_batch(const wind_kv_pool* src, const wind_kv_migrate_item* items,

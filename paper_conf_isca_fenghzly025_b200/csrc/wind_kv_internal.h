@@ -20,8 +20,10 @@ constexpr int kMaxSegs = 32;  // segments (runs) per work unit = one warp's tabl
 struct Item {
   const int32_t* sbt;
   const int32_t* dbt;
-  uint8_t* dst_plane0;     // dst chunk (layer lo, K, block 0)
-  int64_t d_plane_stride;  // NB_dst * C
+  uint8_t* dst_plane0;     // dst chunk (layer lo, K, block 0) + head offset
+  int64_t d_plane_stride;  // NB_dst * C_dst
+  int64_t d_chunk;         // C_dst: block stride inside a dst plane
+  int32_t coalesce;        // runs of adjacent blocks are contiguous on both sides
   uint32_t* flags;         // dst layer_done[0 .. d_layers)
   int32_t d_flag_lo;       // index of global layer lo in flags
   int32_t d_layers;        // dst n_layers (for the out-of-range increments)
@@ -32,9 +34,10 @@ struct Item {
 };
 
 struct Params {
-  const uint8_t* src_plane0;  // src chunk (layer lo, K, block 0)
-  int64_t s_plane_stride;     // NB_src * C
-  int64_t chunk;              // C
+  const uint8_t* src_plane0;  // src chunk (layer lo, K, block 0) + head offset
+  int64_t s_plane_stride;     // NB_src * C_src
+  int64_t s_chunk;            // C_src: block stride inside a src plane
+  int64_t copy;               // bytes copied per (layer, kv, block): C, or n_heads * tile
   int64_t units_per_plane;    // sum of items' units
   int64_t total_units;        // planes * units_per_plane
   uint32_t* counters;         // this op's counter slot, [hi - lo]

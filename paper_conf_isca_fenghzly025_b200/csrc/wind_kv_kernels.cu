@@ -186,18 +186,18 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
   r -= it.unit_base;
   const uint8_t* splane = p.src_plane0 + plane * p.s_plane_stride;
   uint8_t* dplane = it.dst_plane0 + plane * it.d_plane_stride;
-  const int64_t C = p.chunk;
+  const int64_t CS = p.s_chunk, CD = it.d_chunk, CP = p.copy;  // CP == CS == CD unless a head range
   *plane_out = static_cast<int32_t>(plane);
-  if (p.parts > 1) {  // one chunk, piece `part`
+  if (p.parts > 1) {  // one block's span, piece `part`
     const int32_t i = r / p.parts;
     const int32_t part = r - i * p.parts;
     const int64_t off = static_cast<int64_t>(part) * p.part_bytes;
-    const int64_t rest = C - off;
+    const int64_t rest = CP - off;
     const uint32_t len = static_cast<uint32_t>(rest < p.part_bytes ? rest : p.part_bytes);
     if (lane == 0) {
       const int32_t s = it.sbt[i], d = it.dbt[i];
-      segs[0].src = splane + s * C + off;
-      segs[0].dst = dplane + d * C + off;
+      segs[0].src = splane + s * CS + off;
+      segs[0].dst = dplane + d * CD + off;
       segs[0].len = len;
       segs[0].soff = 0;
     }
@@ -214,18 +214,18 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
   }
   const int32_t ps = __shfl_up_sync(kFull, s, 1);
   const int32_t pd = __shfl_up_sync(kFull, d, 1);
-  const bool head = lane < cnt && (lane == 0 || !(s == ps + 1 && d == pd + 1));
+  const bool head = lane < cnt && (lane == 0 || !(it.coalesce && s == ps + 1 && d == pd + 1));
   const uint32_t heads = __ballot_sync(kFull, head);
   if (head) {
     const int k = __popc(heads & ((1u << lane) - 1u));       // prefix popcount
     const uint32_t later = heads & ~((2u << lane) - 1u);     // heads after this lane
     const int end = later ? __ffs(later) - 1 : cnt;
-    segs[k].src = splane + s * C;
-    segs[k].dst = dplane + d * C;
-    segs[k].len = static_cast<uint32_t>((end - lane) * C);
-    segs[k].soff = static_cast<uint32_t>(lane * C);
+    segs[k].src = splane + s * CS;
+    segs[k].dst = dplane + d * CD;
+    segs[k].len = static_cast<uint32_t>((end - lane) * CP);
+    segs[k].soff = static_cast<uint32_t>(lane * CP);
   }
-  *bytes_out = static_cast<uint32_t>(cnt * C);
+  *bytes_out = static_cast<uint32_t>(cnt * CP);
   return __popc(heads);
 }
 
