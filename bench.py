@@ -257,7 +257,7 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
     pb = payload_bytes(len(csrc), sh5.n_layers, sh5.chunk_bytes)
     # compaction is idempotent under repetition only for the first run; moving the same
     # pairs again re-copies identical bytes (same traffic), which is what is timed
-    ms = time_device(lambda: wk.compact(pool, ts, td, stream=s), steps, warmup, s) / steps
+    ms = time_device(lambda: wk.compact(pool, ts, td, stream=s), 5 * steps, warmup, s) / (5 * steps)
     gbs = pb / ms / 1e6
     out["c5_compact"] = {"gbs": round(gbs, 1), "hbm_frac": round(2 * gbs / hbm, 3), "ms": round(ms, 3),
                          "moves": int(len(csrc)), "pool_gib": round(pool.nbytes / GiB, 2)}
@@ -295,7 +295,91 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
 
     # (6) stall-free rescheduling of P:120's request (NEXT-1)
     out["stall_free"] = run_stall_free(wk, device)
+    torch.cuda.empty_cache()
+
+    # (7) layer-streamed hand-off overlapped with a running prefill (NEXT-2)
+    out["prefill_overlap_handoff"] = run_handoff(wk, device)
     return out
+
+
+def run_handoff(wk, device, cap_ctas: int = 16, n_tokens: int = 2048, reps: int = 5) -> dict:
+    """NEXT-2 (P:81, P:339, P:353 "overlapping KV transfers with prefill computation"): an
+    OPT-13B prefill of one 2048-token request runs layer by layer (the 24*N*H^2 GEMM FLOPs
+    of Table 1 per layer, as bf16 cuBLAS matmuls on the prefill stream); as soon
+    as layer l is computed, an event releases migrate(layer l) on the migration stream, and
+    the decode side waits on layer_done[l].  Reported: prefill slowdown caused by the
+    overlapped transfer, and the hand-off latency (prefill end -> last layer landed)
+    overlapped vs. transferring everything after the prefill.  Migration capped at
+    `cap_ctas` CTAs (~NVLink rate)."""
+    import torch
+    from windgen import SHAPES
+    sh = SHAPES["C2"]
+    H = sh.n_kv_heads * sh.head_dim  # hidden size 5120
+    L, bs = sh.n_layers, sh.block_size
+    dev = torch.device("cuda", device)
+    nblk = -(-n_tokens // bs)
+    src = make_pool(wk, sh, nblk + 8, device, 1, 1)
+    dst = make_pool(wk, sh, nblk + 8, device, 1, 2)
+    sbt = torch.arange(nblk, dtype=torch.int32, device=dev)
+    dbt = torch.arange(8, 8 + nblk, dtype=torch.int32, device=dev)
+    x = torch.randn(n_tokens, H, device=dev, dtype=torch.bfloat16)
+    w_qkv = torch.randn(H, 3 * H, device=dev, dtype=torch.bfloat16) * 0.01
+    w_o = torch.randn(H, H, device=dev, dtype=torch.bfloat16) * 0.01
+    w_1 = torch.randn(H, 4 * H, device=dev, dtype=torch.bfloat16) * 0.01
+    w_2 = torch.randn(4 * H, H, device=dev, dtype=torch.bfloat16) * 0.01
+    pre, mig, cons = torch.cuda.Stream(device), torch.cuda.Stream(device), torch.cuda.Stream(device)
+    saved = wk.get_tuning(wk.PATH_INTRA)
+    wk.set_tuning(wk.PATH_INTRA, **{**saved, "max_ctas": cap_ctas})
+
+    def layer_compute():
+        with torch.cuda.stream(pre):
+            qkv = x @ w_qkv
+            a = qkv[:, :H] @ w_o
+            h = a @ w_1
+            return h @ w_2
+
+    def run(mode: str):
+        """mode: 'alone' (prefill only), 'overlap' (per-layer migration), 'serial'."""
+        evs = [torch.cuda.Event() for _ in range(L)]
+        t_start, t_pre_end, t_landed = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+        torch.cuda.synchronize()
+        t_start.record(pre)
+        for l in range(L):
+            layer_compute()
+            evs[l].record(pre)
+            if mode == "overlap":
+                mig.wait_event(evs[l])
+                wk.migrate(src, sbt, dst, dbt, layer_lo=l, layer_hi=l + 1, stream=mig)
+        t_pre_end.record(pre)
+        if mode == "serial":
+            mig.wait_event(evs[L - 1])
+            wk.migrate(src, sbt, dst, dbt, stream=mig)
+        if mode != "alone":
+            t = dst.layer_ticket()
+            for l in range(L):
+                wk.layer_wait(dst, l, t, stream=cons)
+            t_landed.record(cons)
+        torch.cuda.synchronize()
+        pre_ms = t_start.elapsed_time(t_pre_end)
+        land = t_pre_end.elapsed_time(t_landed) if mode != "alone" else 0.0
+        return pre_ms, land
+
+    for _ in range(2):
+        run("overlap")
+    res = {}
+    for mode in ("alone", "overlap", "serial"):
+        vals = [run(mode) for _ in range(reps)]
+        res[mode] = (float(np.median([v[0] for v in vals])), float(np.median([v[1] for v in vals])))
+    wk.set_tuning(wk.PATH_INTRA, **saved)
+    flops = 24 * n_tokens * H * H * L
+    return {"request_tokens": n_tokens, "cap_ctas": cap_ctas,
+            "prefill_ms_alone": round(res["alone"][0], 3),
+            "prefill_tflops_alone": round(flops / res["alone"][0] / 1e9, 1),
+            "prefill_ms_with_overlapped_transfer": round(res["overlap"][0], 3),
+            "prefill_slowdown": round(res["overlap"][0] / res["alone"][0] - 1, 4),
+            "handoff_latency_ms_overlapped": round(res["overlap"][1], 3),
+            "handoff_latency_ms_serial": round(res["serial"][1], 3),
+            "kv_bytes": payload_bytes(nblk, L, sh.chunk_bytes)}
 
 
 def run_stall_free(wk, device, cap_ctas: int = 16) -> dict:
@@ -371,7 +455,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:
     bt = perm.view(B, ctx_len // bs).to(dev)
     ctx = torch.full((B,), ctx_len, dtype=torch.int32, device=dev)
     q = torch.randn(B, sh.n_kv_heads, sh.head_dim, device=dev, dtype=torch.float16)
-    bps = 32
+    bps = 64  # sweep r01: 0.978 of HBM on this shape
     scratch = torch.empty(victim.scratch_floats(B, sh.n_kv_heads, ctx_len // bs, bps), device=dev)
     out = torch.empty(B, sh.n_kv_heads, sh.head_dim, device=dev)
     plane = nbv * sh.chunk_bytes
@@ -411,7 +495,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:
     dbt = torch.as_tensor(case.dst_bt, device=dev)
     pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
     saved = wk.get_tuning(wk.PATH_INTRA)
-    for cap in (8, 16, 0):
+    for cap in (2, 4, 8, 16, 0):
         wk.set_tuning(wk.PATH_INTRA, **{**saved, "max_ctas": cap})
         t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, stream=lo_s), 2, 3, lo_s) / 2
         k = int(math.ceil(n_victim_steps * t_alone * 3.0 / t_mig)) + 2
@@ -428,6 +512,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:
         t_with = float(np.median(with_mig))
         res[f"cap{cap or 'none'}"] = {
             "migration_gbs_alone": round(pb / t_mig / 1e6, 1),
+            "migration_hbm_share": round(2 * pb / t_mig / 1e6 / peaks["hbm_gbs"], 4),
             "victim_ms_with_migration": round(t_with, 3),
             "slowdown": round(t_with / t_alone - 1.0, 4),
             "migration_covered_all_victim_steps": bool(covered)}

@@ -128,7 +128,7 @@ std::mutex g_tune_mu;
 wind_kv_tuning g_tune[3] = {
     /* INTRA */ {kTma, 1, 49152, 4, 0, 0, 2},  // sweep r01: 0.998 (C2) / 0.985 (C5) of HBM copy
     /* PEER  */ {kSimt, 4, 32768, 6, 0, 0, 0},
-    /* HOST  */ {kSimt, 4, 32768, 6, 0, 0, 0},
+    /* HOST  */ {kTma, 1, 49152, 4, 64, 0, 2},  // PCIe-bound: 64 SMs reach the link rate
 };
 
 }  // namespace

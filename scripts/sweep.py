@@ -41,8 +41,108 @@ def timeit(fn, stream, reps=10, warm=3):
     return a.elapsed_time(b) / reps
 
 
+def host_sweep():
+    """Host swap path: C1 and C4 geometries, swap_out / swap_in, kernel x CTAs x unit."""
+    s = torch.cuda.Stream(dev)
+    for name, sh, nblk in [("C1", SHAPES["C1"], 256), ("C4", SHAPES["C4"], 512)]:
+        dpool = pool(sh, nblk + 10, 1)
+        hpool = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes,
+                        nblk, loc="host")
+        bt = torch.randperm(nblk + 10)[:nblk].to(torch.int32).to(dev)
+        hbt = torch.arange(nblk, dtype=torch.int32, device=dev)
+        pb = 2 * sh.n_layers * nblk * sh.chunk_bytes
+        for cfg in [dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768),
+                    dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=2, stage_bytes=32768),
+                    dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=65536),
+                    dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=131072),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=32768, stages=6),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=2, stage_bytes=16384, stages=6),
+                    dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768, max_ctas=64),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, max_ctas=64)]:
+            wk.set_tuning(wk.PATH_HOST, **cfg)
+            mo = timeit(lambda: wk.swap_out(dpool, bt, hpool, hbt, stream=s), s, reps=5)
+            mi = timeit(lambda: wk.swap_in(hpool, hbt, dpool, bt, stream=s), s, reps=5)
+            print(json.dumps(dict(case=name, mode="host", **cfg, out_gbs=round(pb / mo / 1e6, 2),
+                                  in_gbs=round(pb / mi / 1e6, 2))), flush=True)
+        hb = torch.empty(pb, dtype=torch.uint8, pin_memory=True)
+        db = torch.empty(pb, dtype=torch.uint8, device=dev)
+        cs = torch.cuda.current_stream(dev)
+        d2h = timeit(lambda: hb.copy_(db, non_blocking=True), cs, reps=5)
+        h2d = timeit(lambda: db.copy_(hb, non_blocking=True), cs, reps=5)
+        print(json.dumps(dict(case=name, mode="copy_engine", d2h_gbs=round(pb / d2h / 1e6, 2),
+                              h2d_gbs=round(pb / h2d / 1e6, 2))), flush=True)
+        del dpool, hpool
+
+
+def victim_check():
+    import victim
+    from windgen import SHAPES as SH
+    sh = SH["C3"]
+    B, ctx_len, bs = 16, 2048, 16
+    nbv = B * ctx_len // bs
+    vp = wk.Pool(8, sh.n_kv_heads, sh.head_dim, bs, 2, nbv)
+    vt = vp.tensor().view(torch.float16)
+    vt.normal_()
+    bt = torch.randperm(nbv).to(torch.int32).view(B, -1).to(dev)
+    ctx = torch.full((B,), ctx_len, dtype=torch.int32, device=dev)
+    q = torch.randn(B, sh.n_kv_heads, 128, device=dev, dtype=torch.float16)
+    plane = nbv * sh.chunk_bytes
+    for bps in (16, 32, 64):
+        scratch = torch.empty(victim.scratch_floats(B, sh.n_kv_heads, ctx_len // bs, bps), device=dev)
+        out = torch.empty(B, sh.n_kv_heads, 128, device=dev)
+        s = torch.cuda.current_stream(dev)
+
+        def step():
+            for l in range(8):
+                kp = vp.base + 2 * l * plane
+                victim.decode_attention(q, kp, kp + plane, bt, ctx, sh.n_kv_heads, bs, scratch, out,
+                                        blocks_per_split=bps, stream=s.cuda_stream)
+        ms = timeit(step, s, reps=10)
+        kv = 8 * 2 * B * ctx_len * sh.n_kv_heads * 128 * 2
+        print(json.dumps(dict(mode="victim", blocks_per_split=bps, ms=round(ms, 3),
+                              hbm_frac=round(kv / ms / 1e6 / PEAK, 3))), flush=True)
+
+
+def compact_sweep():
+    """C5 compaction (same pool, fp8, C = 16 KiB) over TMA / SIMT configurations."""
+    from windgen import request_lengths, skewed_placement, blocks_for_tokens, live_mask_after_free
+    sh5 = SHAPES["C5"]
+    lens = request_lengths("C5")
+    place = skewed_placement(lens.size, 8, 4005)
+    reqb = blocks_for_tokens(lens[place == 0], 16)
+    nb = math.ceil(int(reqb.sum()) * 1.1)
+    live, _ = live_mask_after_free(nb, reqb, 0.5, 4006)
+    cs, cd = wk.plan_compact(live)
+    runs = 1 + int(np.sum((np.diff(cs) != 1) | (np.diff(cd) != 1)))
+    p = pool(sh5, nb, 1)
+    ts, td = torch.as_tensor(cs, device=dev), torch.as_tensor(cd, device=dev)
+    pb = 2 * sh5.n_layers * len(cs) * sh5.chunk_bytes
+    s = torch.cuda.Stream(dev)
+    print(json.dumps(dict(mode="compact_info", moves=len(cs), runs=runs, pool_blocks=nb)), flush=True)
+    for cfg in [dict(kernel=wk.KERNEL_TMA, stage_bytes=49152, stages=4, ctas_per_sm=1, store_lag=2),
+                dict(kernel=wk.KERNEL_TMA, stage_bytes=32768, stages=6, ctas_per_sm=1, store_lag=3),
+                dict(kernel=wk.KERNEL_TMA, stage_bytes=32768, stages=6, ctas_per_sm=1, store_lag=2),
+                dict(kernel=wk.KERNEL_TMA, stage_bytes=16384, stages=6, ctas_per_sm=2, store_lag=3),
+                dict(kernel=wk.KERNEL_TMA, stage_bytes=16384, stages=12, ctas_per_sm=1, store_lag=6),
+                dict(kernel=wk.KERNEL_TMA, stage_bytes=65536, stages=3, ctas_per_sm=1, store_lag=1),
+                dict(kernel=wk.KERNEL_SIMT, stage_bytes=32768, ctas_per_sm=4),
+                dict(kernel=wk.KERNEL_SIMT, stage_bytes=65536, ctas_per_sm=2)]:
+        wk.set_tuning(wk.PATH_INTRA, **cfg)
+        ms = timeit(lambda: wk.compact(p, ts, td, stream=s), s, reps=10)
+        gbs = pb / ms / 1e6
+        print(json.dumps(dict(case="C5compact", **cfg, ms=round(ms, 3), gbs=round(gbs, 1),
+                              frac=round(2 * gbs / PEAK, 4))), flush=True)
+
+
 def main():
     which = sys.argv[1] if len(sys.argv) > 1 else "all"
+    if which == "host":
+        return host_sweep()
+    if which == "compact":
+        return compact_sweep()
+    if which == "victim":
+        return victim_check()
     s = torch.cuda.Stream(dev)
     out = []
     cases = {}

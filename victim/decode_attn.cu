@@ -23,12 +23,6 @@ struct Partial {
   float m, s;
 };
 
-__device__ __forceinline__ float warp_sum(float v) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
-  return v;
-}
-
 // grid: (B * Hq, splits); block: kWarps warps.  Each warp walks blocks of its split
 // round-robin, keeps an online softmax over its tokens, then the CTA merges its warps.
 __global__ void __launch_bounds__(kWarps * 32) decode_split_kernel(
@@ -48,40 +42,95 @@ __global__ void __launch_bounds__(kWarps * 32) decode_split_kernel(
   const size_t tile = static_cast<size_t>(bs) * kD * sizeof(__half);  // one head tile
   const size_t chunk = static_cast<size_t>(hkv) * tile;               // one block chunk
 
-  const __half2* qh = reinterpret_cast<const __half2*>(q + (static_cast<size_t>(b) * hq + h) * kD) + lane * 2;
-  const float2 q01 = __half22float2(qh[0]);
-  const float2 q23 = __half22float2(qh[1]);
-  float m = -INFINITY, s = 0.f, a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
+  // Lane layout: half-warp `hw` (= lane / 16) takes the tokens of parity hw; lane `dl` (=
+  // lane % 16) holds dims [8 dl, 8 dl + 8) as one 16-B vector, so one warp-wide load moves
+  // two adjacent 256-B token rows.  Each half-warp keeps its own online softmax; the two
+  // are merged after the loop.
+  const int hw = lane >> 4, dl = lane & 15;
+  const uint4 qv = *reinterpret_cast<const uint4*>(q + (static_cast<size_t>(b) * hq + h) * kD + dl * 8);
+  float qf[8];
+  {
+    const __half2* q2 = reinterpret_cast<const __half2*>(&qv);
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const float2 f = __half22float2(q2[j]);
+      qf[2 * j] = f.x * scale;
+      qf[2 * j + 1] = f.y * scale;
+    }
+  }
+  float m = -INFINITY, s = 0.f, acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
 
   for (int blk = blk0 + warp; blk < blk1; blk += kWarps) {
     const int slot = bt[static_cast<size_t>(b) * max_blocks + blk];
     const uint8_t* kt = k_plane + slot * chunk + hk * tile;
     const uint8_t* vt = v_plane + slot * chunk + hk * tile;
     const int ntok = min(bs, len - blk * bs);
-    uint2 kr[kBs], vr[kBs];
+    uint4 kr[kBs / 2], vr[kBs / 2];
 #pragma unroll
-    for (int t = 0; t < kBs; ++t)
-      if (t < ntok) kr[t] = *reinterpret_cast<const uint2*>(kt + t * kD * 2 + lane * 8);
-#pragma unroll
-    for (int t = 0; t < kBs; ++t)
-      if (t < ntok) vr[t] = *reinterpret_cast<const uint2*>(vt + t * kD * 2 + lane * 8);
-#pragma unroll
-    for (int t = 0; t < kBs; ++t) {
-      if (t >= ntok) break;
-      const float2 k01 = __half22float2(*reinterpret_cast<const __half2*>(&kr[t].x));
-      const float2 k23 = __half22float2(*reinterpret_cast<const __half2*>(&kr[t].y));
-      const float x = warp_sum(q01.x * k01.x + q01.y * k01.y + q23.x * k23.x + q23.y * k23.y) * scale;
-      const float mn = fmaxf(m, x);
-      const float c = __expf(m - mn), p = __expf(x - mn);
-      const float2 v01 = __half22float2(*reinterpret_cast<const __half2*>(&vr[t].x));
-      const float2 v23 = __half22float2(*reinterpret_cast<const __half2*>(&vr[t].y));
-      s = s * c + p;
-      a0 = a0 * c + p * v01.x;
-      a1 = a1 * c + p * v01.y;
-      a2 = a2 * c + p * v23.x;
-      a3 = a3 * c + p * v23.y;
-      m = mn;
+    for (int t2 = 0; t2 < kBs / 2; ++t2) {
+      const int t = 2 * t2 + hw;
+      if (t < ntok) kr[t2] = *reinterpret_cast<const uint4*>(kt + t * kD * 2 + dl * 16);
     }
+#pragma unroll
+    for (int t2 = 0; t2 < kBs / 2; ++t2) {
+      const int t = 2 * t2 + hw;
+      if (t < ntok) vr[t2] = *reinterpret_cast<const uint4*>(vt + t * kD * 2 + dl * 16);
+    }
+#pragma unroll
+    for (int t2 = 0; t2 < kBs / 2; ++t2) {
+      const int t = 2 * t2 + hw;
+      const __half2* k2 = reinterpret_cast<const __half2*>(&kr[t2]);
+      float x = 0.f;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const float2 f = __half22float2(k2[j]);
+        x += qf[2 * j] * f.x + qf[2 * j + 1] * f.y;
+      }
+#pragma unroll
+      for (int o = 8; o > 0; o >>= 1) x += __shfl_xor_sync(0xffffffffu, x, o);  // within the half
+      if (t < ntok) {
+        const float mn = fmaxf(m, x);
+        const float c = __expf(m - mn), p = __expf(x - mn);
+        const __half2* v2 = reinterpret_cast<const __half2*>(&vr[t2]);
+        s = s * c + p;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const float2 f = __half22float2(v2[j]);
+          acc[2 * j] = acc[2 * j] * c + p * f.x;
+          acc[2 * j + 1] = acc[2 * j + 1] * c + p * f.y;
+        }
+        m = mn;
+      }
+    }
+  }
+  // merge the two half-warps (token parities): lane dl of half 0 with lane dl of half 1
+  {
+    const float mo = __shfl_xor_sync(0xffffffffu, m, 16);
+    const float so = __shfl_xor_sync(0xffffffffu, s, 16);
+    const float M = fmaxf(m, mo);
+    const float c1 = (m == -INFINITY) ? 0.f : __expf(m - M);
+    const float c2 = (mo == -INFINITY) ? 0.f : __expf(mo - M);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float ao = __shfl_xor_sync(0xffffffffu, acc[j], 16);
+      acc[j] = acc[j] * c1 + ao * c2;
+    }
+    s = s * c1 + so * c2;
+    m = M;
+  }
+  // lane dl of half 0 now holds dims [8 dl, 8 dl + 8); write as the 4-per-lane layout below
+  float a0, a1, a2, a3;
+  {
+    // lane L needs dims [4L, 4L + 4) = half (L & 1) of lane (L >> 1)'s 8 dims
+    const int srcl = lane >> 1;
+    float g[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) g[j] = __shfl_sync(0xffffffffu, acc[j], srcl);
+    const bool hi4 = lane & 1;
+    a0 = hi4 ? g[4] : g[0];
+    a1 = hi4 ? g[5] : g[1];
+    a2 = hi4 ? g[6] : g[2];
+    a3 = hi4 ? g[7] : g[3];
   }
   // merge the CTA's warps
   __shared__ float sm_m[kWarps], sm_s[kWarps];
