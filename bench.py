@@ -36,6 +36,8 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "KV migration GB/s (fraction of NVLink/HBM roofline) at 1/2/4/8 B200"
+LENGTH_MIX = {"C1": "512 tok each", "C2": "ShareGPT-fit 256-2048 tok", "C3": "2048 tok each",
+              "C4": "LongBench-fit 16-4096 tok", "C5": "long-tail lognormal 16-8192 tok"}
 GiB = 1 << 30
 
 
@@ -521,7 +523,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:
     return res
 
 
-def run_all_to_all(wk, rank, world, device, peaks, steps=5, warmup=3) -> dict:
+def run_all_to_all(wk, rank, world, device, peaks, steps=5, warmup=3, scale=1.0) -> dict:
     """A8 at N > 1: C5 (Llama-3-8B GQA fp8, 1024 long-tail requests) placed with skewed
     weights over the ranks; every rank derives the same plan (uniform hash shuffle =
     bandwidth headline; greedy rebalance = realistic), imports every peer's pool and pushes
@@ -532,7 +534,7 @@ def run_all_to_all(wk, rank, world, device, peaks, steps=5, warmup=3) -> dict:
     from windgen import (SHAPES, request_lengths, skewed_placement, blocks_for_tokens,
                          hash_shuffle_dest)
     sh = SHAPES["C5"]
-    lens = request_lengths("C5")
+    lens = request_lengths("C5", scale=scale)
     gpu = skewed_placement(lens.size, world, 4005)
     blocks = blocks_for_tokens(lens, 16).astype(np.int32)
     loads = np.bincount(gpu, weights=blocks, minlength=world).astype(np.int64)
@@ -601,6 +603,8 @@ def run_gpu(args) -> None:
     rank = int(os.environ.get("RANK", 0))
     world = int(os.environ.get("WORLD_SIZE", 1))
     local = int(os.environ.get("LOCAL_RANK", 0))
+    if os.environ.get("WIND_BENCH_ONE_DEVICE"):  # test hook: every rank on cuda:0 (CUDA IPC
+        local = 0                                 # between processes on one GPU)
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
     torch.cuda.set_device(local)
@@ -666,7 +670,7 @@ def run_gpu(args) -> None:
     if world > 1 and args.scenarios:
         del src, dst
         torch.cuda.empty_cache()
-        a2a = run_all_to_all(wk, rank, world, local, peaks)
+        a2a = run_all_to_all(wk, rank, world, local, peaks, scale=args.a2a_scale)
     value = total_bytes / ms_step / 1e6  # GB/s
     e2e_value = total_bytes / ms_e2e / 1e6
 
@@ -700,7 +704,7 @@ def run_gpu(args) -> None:
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u8", "data": "synthetic",
             "config": {"workload": f"{args.config} {sh.name} KV: {case.n} blocks of {case.lengths.size} "
-                                   f"requests (ShareGPT-fit 256-2048 tok), {args.variant} tables, "
+                                   f"requests ({LENGTH_MIX.get(args.config, '')}), {args.variant} tables, "
                                    f"prefill pool -> decode pool, layers 0-{sh.n_layers - 1}",
                        "payload_gib_per_pair": round(pb / GiB, 3),
                        "placement": "same GPU" if world == 1 else "pairs 2k->2k+1 over NVLink peer stores",
@@ -777,6 +781,8 @@ def main():
     ap.add_argument("--scenarios", dest="scenarios", action="store_true", default=True)
     ap.add_argument("--no-scenarios", dest="scenarios", action="store_false")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--a2a-scale", type=float, default=1.0,
+                    help="request-count scale of the N>1 all-to-all scenario (C5 = 1.0)")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
