@@ -494,6 +494,11 @@ wind_status route(const wind_kv_pool* src, const wind_kv_pool* dst, int* exec, i
 
 wind_status check_stream(void* stream, int exec) {
   if (!stream) return WIND_OK;  // legacy default stream of the executing device
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(static_cast<cudaStream_t>(stream), &cap) == cudaSuccess &&
+      cap != cudaStreamCaptureStatusNone)
+    return WIND_OK;  // cudaStreamGetDevice is not permitted while capturing; trust the caller
+  cudaGetLastError();
   int sd = -1;
   cudaError_t e = cudaStreamGetDevice(static_cast<cudaStream_t>(stream), &sd);
   if (e != cudaSuccess) {

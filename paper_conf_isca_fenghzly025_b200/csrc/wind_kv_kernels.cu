@@ -309,7 +309,7 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
 
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
-      mbar_init(&full[i], 1);
+      mbar_init(&full[i], 32);  // every producer lane arrives: each releases its own segment writes
       mbar_init(&empty[i], 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -325,16 +325,15 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
       const int st = it % S;
       if (it >= S) mbar_wait(&empty[st], ((it / S) & 1) ^ 1);
       if (u >= total) {
-        if (lane == 0) {
-          desc[st].nseg = -1;
-          mbar_arrive(&full[st]);
-        }
+        if (lane == 0) desc[st].nseg = -1;
+        mbar_arrive(&full[st]);
         break;
       }
       int32_t plane;
       uint32_t bytes;
       const int nseg = decode_unit(p, u, desc[st].segs, &plane, &bytes);
       __syncwarp();
+      if (lane != 0) mbar_arrive(&full[st]);
       if (lane == 0) {
         desc[st].nseg = nseg;
         desc[st].plane = plane;

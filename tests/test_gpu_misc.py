@@ -1,0 +1,91 @@
+"""GPU: CUDA-graph capture of the ops, external pool bases, and launch accounting."""
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+import paper_conf_isca_fenghzly025_b200 as wk
+from windgen import migration_case, KVShape
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda", 0)
+
+
+def geom(p):
+    d = p.desc
+    return O.Geom(d.first_layer, d.n_layers, d.n_kv_heads, d.head_dim, d.block_size, d.elem_bytes,
+                  d.n_blocks)
+
+
+def test_migrate_is_graph_capturable():
+    """wind_kv.h: ops never allocate or synchronise, so they can be captured in a CUDA
+    graph and replayed (the layer flags count every replay)."""
+    case = migration_case("C1", scale=0.5)
+    sh = case.shape
+    src = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, case.nb_src)
+    dst = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, case.nb_dst)
+    rng = np.random.default_rng(0)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    d0 = rng.integers(0, 256, dst.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    dst.tensor().copy_(torch.from_numpy(d0))
+    ts = torch.as_tensor(case.src_bt, device=DEV)
+    td = torch.as_tensor(case.dst_bt, device=DEV)
+    s = torch.cuda.Stream(DEV)
+    torch.cuda.synchronize()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=s):
+        wk.migrate(src, ts, dst, td, layer_lo=2, layer_hi=9, stream=s)
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(dst.tensor().cpu().numpy(), d0)  # capture ran nothing
+    for _ in range(3):
+        g.replay()
+    torch.cuda.synchronize()
+    want = d0.copy()
+    assert O.migrate(s0, geom(src), case.src_bt, want, geom(dst), case.dst_bt, 2, 9) == O.OK
+    np.testing.assert_array_equal(dst.tensor().cpu().numpy(), want)
+    assert all(dst.layer_count(l) == 3 for l in range(sh.n_layers))
+
+
+def test_external_base_pools():
+    """Pools over caller memory (torch allocations): used in place, never freed by the
+    library; a misaligned base is INVALID_ARG."""
+    sh = KVShape("t", 2, 4, 64, 2)
+    nb = 30
+    nbytes = sh.n_layers * 2 * nb * sh.chunk_bytes
+    buf_s = torch.randint(0, 256, (nbytes,), dtype=torch.uint8, device=DEV)
+    buf_d = torch.randint(0, 256, (nbytes + 16,), dtype=torch.uint8, device=DEV)
+    src = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, nb,
+                  external_base=buf_s.data_ptr())
+    with pytest.raises(wk.WindKVError) as e:
+        wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, nb,
+                external_base=buf_d.data_ptr() + 8)
+    assert e.value.status == -1
+    dst = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, nb,
+                  external_base=buf_d.data_ptr() + 16)
+    assert src.base == buf_s.data_ptr() and dst.base == buf_d.data_ptr() + 16
+    s0, d0 = buf_s.cpu().numpy().copy(), buf_d[16:].cpu().numpy().copy()
+    sbt, dbt = np.array([3, 9, 29, 0], np.int32), np.array([1, 2, 3, 28], np.int32)
+    wk.migrate(src, torch.as_tensor(sbt, device=DEV), dst, torch.as_tensor(dbt, device=DEV))
+    torch.cuda.synchronize()
+    want = d0.copy()
+    g = O.Geom(0, 2, 4, 64, 16, 2, nb)
+    assert O.migrate(s0, g, sbt, want, g, dbt, 0, 2) == O.OK
+    np.testing.assert_array_equal(buf_d[16:].cpu().numpy(), want)
+    src.destroy()
+    dst.destroy()
+    assert buf_s.sum().item() >= 0  # caller memory still valid after destroy
+
+
+def test_launch_count_one_kernel_per_op():
+    sh = KVShape("t", 2, 4, 64, 2)
+    a = wk.Pool(2, 4, 64, 16, 2, 20)
+    b = wk.Pool(2, 4, 64, 16, 2, 20)
+    t = torch.arange(10, dtype=torch.int32, device=DEV)
+    n0 = wk.launch_count()
+    for _ in range(7):
+        wk.migrate(a, t, b, t)
+    wk.migrate_batch(a, [(b, t, t)], 0, 2)
+    torch.cuda.synchronize()
+    assert wk.launch_count() - n0 == 8
+    del sh
