@@ -244,6 +244,20 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
     gbs = pb / ms / 1e6
     out["c2_layer_streamed"] = {"gbs": round(gbs, 1), "hbm_frac": round(2 * gbs / hbm, 3),
                                 "ms": round(ms, 3), "launches_per_step": sh.n_layers}
+
+    # copy-engine comparators on the same C2 gather (S§7 step 4): per-chunk cudaMemcpyAsync
+    # (the classic per-block swap loop) and cudaMemcpyBatchAsync; host tables
+    import victim
+    planes = 2 * sh.n_layers
+    for kind, st in (("loop", 1), ("batch", 2)):
+        def ce():
+            victim.ce_gather(kind, src.base, case.nb_src * sh.chunk_bytes, dst.base,
+                             case.nb_dst * sh.chunk_bytes, sh.chunk_bytes, case.src_bt, case.dst_bt,
+                             planes, s.cuda_stream)
+        ms = time_device(ce, st, 3 if kind == "batch" else 1 + 2, s) / st
+        gbs = pb / ms / 1e6
+        out[f"c2_copy_engine_{kind}"] = {"gbs": round(gbs, 1), "hbm_frac": round(2 * gbs / hbm, 3),
+                                         "ms": round(ms, 3), "copies": planes * case.n}
     del src, dst
 
     # (3) C5 compaction on GPU 0's share of the skewed placement (A7)
@@ -689,11 +703,13 @@ def run_gpu(args) -> None:
                     "frac": round(kernel_gbs / 900.0, 4), "traffic": None, "peak_src": "nominal",
                     "per_launch_bytes": pb}
         extra["roofline"] = roof
-        extra["parity"] = parity_sample(wk, case, src, dst, lo, hi) if world == 1 else None
         if a2a is not None:
             extra["scenarios"] = {"c5_all_to_all": a2a}
         if world == 1 and not args.no_cpu_baseline:
+            # the cpu_baseline leg: the oracle timed on the host cores, and (outside every
+            # timed region) the oracle's sampled check of this run's GPU output
             extra["cpu_baseline"] = cpu_baseline(case)
+            extra["cpu_baseline"]["parity_check_of_this_run"] = parity_sample(wk, case, src, dst, lo, hi)
         if world == 1 and args.scenarios:
             del src, dst
             torch.cuda.empty_cache()

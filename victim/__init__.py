@@ -1,25 +1,38 @@
-"""victim — BENCH HARNESS ONLY: paged decode attention over a wind_kv pool, the
-co-running "decode stream" of the interference measurement (S§8(d)).  Not part of the
-product library; validated against torch SDPA in tests/test_gpu_victim.py."""
+"""victim — BENCH HARNESS ONLY, not part of the product library:
+  * paged decode attention over a wind_kv pool: the co-running "decode stream" of the
+    interference measurement (S§8(d)); validated against torch attention in
+    tests/test_gpu_victim.py;
+  * copy-engine comparators (cudaMemcpyAsync per chunk, cudaMemcpyBatchAsync) for the same
+    paged gather (S§7 step 4)."""
 from __future__ import annotations
 
 import ctypes as ct
 import os
 import subprocess
 
+import numpy as np
+
 HERE = os.path.dirname(os.path.abspath(__file__))
 SRC = os.path.join(HERE, "decode_attn.cu")
 LIB = os.path.join(HERE, "libwind_victim.so")
+CE_SRC = os.path.join(HERE, "ce_gather.cu")
+CE_LIB = os.path.join(HERE, "libwind_ce.so")
 _L = None
+_CE = None
+
+
+def _nvcc(src: str, out: str) -> None:
+    tmp = out + f".tmp{os.getpid()}"
+    subprocess.check_call([os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc"), "-gencode",
+                           "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-shared",
+                           "-Xcompiler", "-fPIC", "-o", tmp, src])
+    os.replace(tmp, out)
 
 
 def build(force: bool = False) -> str:
-    if force or not os.path.exists(LIB) or os.path.getmtime(LIB) < os.path.getmtime(SRC):
-        tmp = LIB + f".tmp{os.getpid()}"
-        subprocess.check_call([os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc"), "-gencode",
-                               "arch=compute_100a,code=sm_100a", "-O3", "-lineinfo", "-shared",
-                               "-Xcompiler", "-fPIC", "-o", tmp, SRC])
-        os.replace(tmp, LIB)
+    for src, out in ((SRC, LIB), (CE_SRC, CE_LIB)):
+        if force or not os.path.exists(out) or os.path.getmtime(out) < os.path.getmtime(src):
+            _nvcc(src, out)
     return LIB
 
 
@@ -34,6 +47,21 @@ def _lib():
         f.restype = ct.c_int
         _L = L
     return _L
+
+
+def _ce():
+    global _CE
+    if _CE is None:
+        if not os.path.exists(CE_LIB):
+            raise ImportError(f"{CE_LIB} missing: run __graft_entry__.build()")
+        L = ct.CDLL(CE_LIB)
+        for name in ("ce_gather_loop", "ce_gather_batch"):
+            f = getattr(L, name)
+            f.argtypes = [ct.c_void_p, ct.c_int64, ct.c_void_p, ct.c_int64, ct.c_int64, ct.c_void_p,
+                          ct.c_void_p, ct.c_int32, ct.c_int32, ct.c_void_p]
+            f.restype = ct.c_int
+        _CE = L
+    return _CE
 
 
 def scratch_floats(batch: int, hq: int, max_blocks: int, blocks_per_split: int) -> int:
@@ -52,3 +80,16 @@ def decode_attention(q, k_plane_ptr: int, v_plane_ptr: int, bt, ctx, hkv: int, b
                                         stream or None)
     if rc != 0:
         raise RuntimeError(f"victim_decode_attention failed ({rc})")
+
+
+def ce_gather(kind: str, src_plane0: int, s_stride: int, dst_plane0: int, d_stride: int, chunk: int,
+              src_bt: np.ndarray, dst_bt: np.ndarray, planes: int, stream: int) -> None:
+    """Copy-engine gather: kind 'loop' (cudaMemcpyAsync per chunk) or 'batch'
+    (cudaMemcpyBatchAsync).  Tables are host int32 arrays."""
+    s = np.ascontiguousarray(src_bt, np.int32)
+    d = np.ascontiguousarray(dst_bt, np.int32)
+    f = _ce().ce_gather_loop if kind == "loop" else _ce().ce_gather_batch
+    rc = f(src_plane0, s_stride, dst_plane0, d_stride, chunk, s.ctypes.data, d.ctypes.data, s.size,
+           planes, stream or None)
+    if rc != 0:
+        raise RuntimeError(f"ce_gather_{kind} failed (cudaError {rc})")
