@@ -174,7 +174,8 @@ def _stream(stream, device: int) -> Optional[int]:
 class _CudaArray:
     """__cuda_array_interface__ wrapper so torch can view library-owned device memory."""
 
-    def __init__(self, ptr: int, nbytes: int):
+    def __init__(self, ptr: int, nbytes: int, owner=None):
+        self._owner = owner  # the Pool: kept alive as long as a tensor view exists
         self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1",
                                          "data": (ptr, False), "version": 3}
 
@@ -186,7 +187,6 @@ class Pool:
                  elem_bytes: int, n_blocks: int, *, loc: str = "device", device: int = 0,
                  first_layer: int = 0, debug: bool = False, external_base: Optional[int] = None,
                  _handle: Optional[int] = None):
-        self._owner_ref = None
         if _handle is None:
             d = PoolDesc(first_layer, n_layers, n_kv_heads, head_dim, block_size, elem_bytes,
                          n_blocks, LOC_HOST if loc == "host" else LOC_DEVICE, device,
@@ -234,14 +234,14 @@ class Pool:
             arr = np.ctypeslib.as_array((ct.c_ubyte * self.nbytes).from_address(self.base))
             return torch.from_numpy(arr)
         with torch.cuda.device(self.device):
-            return torch.as_tensor(_CudaArray(self.base, self.nbytes), device=f"cuda:{self.device}")
+            return torch.as_tensor(_CudaArray(self.base, self.nbytes, self), device=f"cuda:{self.device}")
 
     def flags_tensor(self, device: Optional[int] = None):
         """A torch int32 view of layer_done[n_layers] (device-accessible flags)."""
         import torch
         dev = self.device if device is None else device
         with torch.cuda.device(dev):
-            t = torch.as_tensor(_CudaArray(self.flags_ptr, 4 * self.desc.n_layers),
+            t = torch.as_tensor(_CudaArray(self.flags_ptr, 4 * self.desc.n_layers, self),
                                 device=f"cuda:{dev}")
         return t.view(torch.int32)
 

@@ -127,7 +127,10 @@ wind_status dev_ctx(int dev, DevCtx** out) {
 std::mutex g_tune_mu;
 wind_kv_tuning g_tune[3] = {
     /* INTRA */ {kTma, 1, 49152, 4, 0, 0, 2},  // sweep r01: 0.998 (C2) / 0.985 (C5) of HBM copy
-    /* PEER  */ {kSimt, 4, 32768, 6, 0, 0, 0},
+    // PEER: SM stores over NVLink (the path the guide measures at 775 GB/s); 96 CTAs of 512
+    // threads keep ~3 MiB of stores in flight (> 2 us x 900 GB/s) and leave SMs to the
+    // co-running prefill / decode.  Not yet tuned on a multi-GPU box (one GPU per round-1 call).
+    /* PEER  */ {kSimt, 1, 32768, 6, 96, 0, 0},
     /* HOST  */ {kTma, 1, 49152, 4, 64, 0, 2},  // PCIe-bound: 64 SMs reach the link rate
 };
 
