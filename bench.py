@@ -662,7 +662,6 @@ def run_gpu(args) -> None:
     h_dbt = torch.as_tensor(case.dst_bt).pin_memory()
     d_sbt, d_dbt = torch.empty_like(sbt), torch.empty_like(dbt)
     flags_host = torch.empty(sh.n_layers, dtype=torch.int32).pin_memory()
-    flags_dev = dst.flags_tensor(local) if dst is not None else None
 
     def e2e_step():
         if role == "decode":
@@ -671,8 +670,7 @@ def run_gpu(args) -> None:
             d_sbt.copy_(h_sbt, non_blocking=True)
             d_dbt.copy_(h_dbt, non_blocking=True)
         wk.migrate(src, d_sbt, dst, d_dbt, layer_lo=lo, layer_hi=hi, stream=stream)
-        with torch.cuda.stream(stream):
-            flags_host.copy_(flags_dev, non_blocking=True)
+        dst.read_flags(flags_host, stream=stream)  # the step's result: layer_done[] D2H
         stream.synchronize()
 
     ms_e2e_local = time_device(e2e_step, max(3, args.steps // 2), 2, stream, barrier) / max(3, args.steps // 2)

@@ -214,6 +214,11 @@ wind_status wind_kv_layer_ticket(const wind_kv_pool* dst, uint32_t* ticket);
 wind_status wind_kv_layer_wait(const wind_kv_pool* dst, int32_t layer, uint32_t ticket,
                                void* consumer);
 
+/* Asynchronous copy of all n_layers layer_done flags into caller memory `out` (pinned
+ * host or device memory, n_layers uint32) on `stream` (a stream of the pool's local device;
+ * for imported pools the flags are read over the peer mapping).  No host sync. */
+wind_status wind_kv_read_flags(const wind_kv_pool* pool, uint32_t* out, void* stream);
+
 /* Host read of layer_done[layer] (synchronous; tests and diagnostics). */
 wind_status wind_kv_layer_count(const wind_kv_pool* dst, int32_t layer, uint32_t* value);
 

@@ -47,7 +47,7 @@ EXPORTED_SYMBOLS = [
     "wind_kv_pool_export", "wind_kv_pool_import", "wind_kv_migrate", "wind_kv_swap_out",
     "wind_kv_swap_in", "wind_kv_compact", "wind_kv_migrate_batch", "wind_kv_migrate_heads",
     "wind_kv_layer_ticket",
-    "wind_kv_layer_wait", "wind_kv_layer_count", "wind_kv_validate", "wind_kv_plan_compact",
+    "wind_kv_layer_wait", "wind_kv_layer_count", "wind_kv_read_flags", "wind_kv_validate", "wind_kv_plan_compact",
     "wind_kv_plan_rebalance", "wind_kv_check_device_error", "wind_kv_set_tuning",
     "wind_kv_get_tuning", "wind_kv_launch_count", "wind_kv_status_string", "wind_kv_last_error",
     "wind_kv_version",
@@ -111,6 +111,7 @@ def lib() -> ct.CDLL:
         "wind_kv_layer_ticket": [P, ct.POINTER(U32)],
         "wind_kv_layer_wait": [P, I32, U32, P],
         "wind_kv_layer_count": [P, I32, ct.POINTER(U32)],
+        "wind_kv_read_flags": [P, P, P],
         "wind_kv_validate": [P, P, P, P, I32, I32, I32],
         "wind_kv_plan_compact": [P, I32, P, P, P],
         "wind_kv_plan_rebalance": [I32, I32, P, P, P, P],
@@ -250,6 +251,12 @@ class Pool:
         t = ct.c_uint32()
         _check(lib().wind_kv_layer_ticket(self.handle, ct.byref(t)))
         return int(t.value)
+
+    def read_flags(self, out, stream=None) -> None:
+        """wind_kv_read_flags: async copy of layer_done[n_layers] into `out` (a pinned host
+        or device int32/uint32 tensor, or an address) on `stream`."""
+        ptr = out if isinstance(out, int) else out.data_ptr()
+        _check(lib().wind_kv_read_flags(self.handle, ptr, _stream(stream, self.device)))
 
     def layer_count(self, layer: int) -> int:
         v = ct.c_uint32()

@@ -740,6 +740,19 @@ extern "C" wind_status wind_kv_layer_wait(const wind_kv_pool* dst, int32_t layer
   return WIND_OK;
 }
 
+extern "C" wind_status wind_kv_read_flags(const wind_kv_pool* p, uint32_t* out, void* stream) {
+  if (!p || !out) return fail(WIND_ERR_INVALID_ARG, "NULL argument");
+  if (p->desc.loc == WIND_LOC_DEVICE) {
+    wind_status st = check_stream(stream, p->desc.device);
+    if (st != WIND_OK) return st;
+  }
+  DeviceGuard g(p->desc.loc == WIND_LOC_DEVICE ? p->desc.device : 0);
+  WKV_CUDA(cudaMemcpyAsync(out, p->flags, sizeof(uint32_t) * p->desc.n_layers, cudaMemcpyDefault,
+                           static_cast<cudaStream_t>(stream)),
+           "cudaMemcpyAsync(flags)");
+  return WIND_OK;
+}
+
 extern "C" wind_status wind_kv_layer_count(const wind_kv_pool* dst, int32_t layer, uint32_t* value) {
   if (!dst || !value) return fail(WIND_ERR_INVALID_ARG, "NULL argument");
   if (layer < dst->desc.first_layer || layer >= dst->desc.first_layer + dst->desc.n_layers)

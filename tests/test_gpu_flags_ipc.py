@@ -154,11 +154,18 @@ def test_ipc_push_and_pull_between_processes():
         sbt = rng.permutation(120)[:50].astype(np.int32)
         dbt = rng.permutation(90)[:50].astype(np.int32)
         s = torch.cuda.Stream(DEV)
-        wk.migrate(src, torch.as_tensor(sbt, device=DEV), remote, torch.as_tensor(dbt, device=DEV),
-                   layer_lo=1, layer_hi=4, stream=s)
+        # one batched launch pushes into the imported pool AND a local pool (A8 sender side)
+        side = pattern_pool(sh, 70, 9, 4)
+        sb2 = rng.permutation(120)[:40].astype(np.int32)
+        db2 = rng.permutation(70)[:40].astype(np.int32)
+        wk.migrate_batch(src, [(remote, torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)),
+                               (side, torch.as_tensor(sb2, device=DEV), torch.as_tensor(db2, device=DEV))],
+                         1, 4, stream=s)
         t = remote.layer_ticket()
         for l in range(4):
             wk.layer_wait(remote, l, t, stream=s)
+        flags_h = torch.zeros(4, dtype=torch.int32).pin_memory()
+        remote.read_flags(flags_h, stream=s)  # async read of the peer's flags
         # pull: remote -> a local pool
         back = pattern_pool(sh, 60, 9, 3)
         pb = np.arange(10, dtype=np.int32)
@@ -173,7 +180,11 @@ def test_ipc_push_and_pull_between_processes():
         want = content_bytes(9, 2, 0, got.size)
         assert O.migrate(content_bytes(9, 1, 0, src.nbytes), g_src, sbt, want, g_rem, dbt, 1, 4) == O.OK
         np.testing.assert_array_equal(got, want)
-        assert counts == [1, 1, 1, 1]
+        assert counts == [1, 1, 1, 1] and flags_h.tolist() == [1, 1, 1, 1]
+        want_side = content_bytes(9, 4, 0, side.nbytes)
+        assert O.migrate(content_bytes(9, 1, 0, src.nbytes), g_src, sb2, want_side, geom(side), db2,
+                         1, 4) == O.OK
+        np.testing.assert_array_equal(side.tensor().cpu().numpy(), want_side)
         want_b = content_bytes(9, 3, 0, back.nbytes)
         assert O.migrate(want, g_rem, dbt[:10], want_b, geom(back), pb, 0, 4) == O.OK
         torch.cuda.synchronize()
