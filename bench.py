@@ -315,6 +315,10 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
 
     # (7) layer-streamed hand-off overlapped with a running prefill (NEXT-2)
     out["prefill_overlap_handoff"] = run_handoff(wk, device)
+    torch.cuda.empty_cache()
+
+    # (8) C4 memory pressure: evict by swap vs by migration, swap concurrent with hand-off
+    out["c4_pressure"] = run_pressure(wk, device)
     return out
 
 
@@ -396,6 +400,73 @@ def run_handoff(wk, device, cap_ctas: int = 16, n_tokens: int = 2048, reps: int 
             "handoff_latency_ms_overlapped": round(res["overlap"][1], 3),
             "handoff_latency_ms_serial": round(res["serial"][1], 3),
             "kv_bytes": payload_bytes(nblk, L, sh.chunk_bytes)}
+
+
+def run_pressure(wk, device, reps: int = 3) -> dict:
+    """C4 (Llama-2-70B GQA bf16, 32 LongBench-fit requests per pair) under memory pressure
+    (S§8(d)): the decode pool holds resident requests and must take an incoming batch; it
+    can only hold 0.8 x (resident + incoming), so victims (longest first) must
+    leave.  DistServe swaps them to host; WindServe reschedules them to the
+    prefill instance.  Measured: time to evict the victims by swap-out (PCIe)
+    vs by migration (HBM here; NVLink-rate cap 16 CTAs and uncapped), and the incoming
+    hand-off running concurrently with the swap-out (separate links, separate streams)."""
+    import torch
+    from windgen import SHAPES, lengths_longbench, blocks_for_tokens
+    sh = SHAPES["C4"]
+    dev = torch.device("cuda", device)
+    res_b = blocks_for_tokens(lengths_longbench(32, 1004), 16)
+    inc_b = blocks_for_tokens(lengths_longbench(32, 2004), 16)
+    n_res, n_inc = int(res_b.sum()), int(inc_b.sum())
+    cap = int(0.8 * (n_res + n_inc))
+    need = n_res + n_inc - cap
+    order = np.argsort(-res_b, kind="stable")            # longest first, lowest id on ties
+    take = np.cumsum(res_b[order]) < need
+    take[np.argmin(take)] = True                           # the request that crosses `need`
+    victims = order[take]
+    starts = np.concatenate([[0], np.cumsum(res_b)])
+    vic_slots = np.concatenate([np.arange(starts[r], starts[r + 1]) for r in victims]).astype(np.int32)
+    nv = vic_slots.size
+    dpool = make_pool(wk, sh, cap, device, 3004, 1)         # resident in slots [0, n_res)
+    host = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, nv, loc="host")
+    other = make_pool(wk, sh, nv + 8, device, 3004, 2)      # the prefill instance's pool
+    src_inc = make_pool(wk, sh, n_inc + 8, device, 3004, 3)
+    s_swap, s_mig = torch.cuda.Stream(device), torch.cuda.Stream(device)
+    vt = torch.as_tensor(vic_slots, device=dev)
+    ht = torch.arange(nv, dtype=torch.int32, device=dev)
+    free_now = cap - n_res
+    inc_src = torch.arange(n_inc, dtype=torch.int32, device=dev)
+    inc_dst = torch.as_tensor(np.concatenate([np.arange(n_res, cap), vic_slots])[:n_inc].astype(np.int32),
+                              device=dev)
+    vb = payload_bytes(nv, sh.n_layers, sh.chunk_bytes)
+    ib = payload_bytes(n_inc, sh.n_layers, sh.chunk_bytes)
+    t_swap = time_device(lambda: wk.swap_out(dpool, vt, host, ht, stream=s_swap), reps, 2, s_swap) / reps
+    saved = wk.get_tuning(wk.PATH_INTRA)
+    out = {"victims": int(victims.size), "victim_gib": round(vb / GiB, 2), "incoming_gib": round(ib / GiB, 2),
+           "evict_by_swap_ms": round(t_swap, 2), "swap_gbs": round(vb / t_swap / 1e6, 1)}
+    for capc in (16, 0):
+        wk.set_tuning(wk.PATH_INTRA, **{**saved, "max_ctas": capc})
+        t_m = time_device(lambda: wk.migrate(dpool, vt, other, ht, stream=s_mig), reps, 2, s_mig) / reps
+        out[f"evict_by_migration_ms_cap{capc or 'none'}"] = round(t_m, 3)
+    wk.set_tuning(wk.PATH_INTRA, **saved)
+    # concurrent: swap the victims out while the incoming batch lands in the free slots; the
+    # part that needs victim slots waits for the swap-out (an event after swap_out)
+    k_free = min(free_now, n_inc)
+
+    def both():
+        ev = torch.cuda.Event()
+        wk.swap_out(dpool, vt, host, ht, stream=s_swap)
+        ev.record(s_swap)
+        wk.migrate(src_inc, inc_src[:k_free], dpool, inc_dst[:k_free], stream=s_mig)
+        if n_inc > k_free:
+            s_mig.wait_event(ev)
+            wk.migrate(src_inc, inc_src[k_free:], dpool, inc_dst[k_free:], stream=s_mig)
+        s_mig.wait_stream(s_swap)
+    t_both = time_device(both, reps, 1, s_mig) / reps
+    out["swap_out_plus_incoming_ms"] = round(t_both, 2)
+    out["paper_claim"] = ("rescheduling (migration) instead of swapping frees the decode pool "
+                          f"{t_swap / out['evict_by_migration_ms_cap16']:.0f}x faster at an NVLink-rate cap")
+    del dpool, host, other, src_inc
+    return out
 
 
 def run_stall_free(wk, device, cap_ctas: int = 16) -> dict:
