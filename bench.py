@@ -515,7 +515,7 @@ def run_stall_free(wk, device, cap_ctas: int = 16) -> dict:
             "blocks_sent": res.blocks_sent}
 
 
-def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:
+def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict:
     """S§8(d) interference, C3 (OPT-66B KV, 64 layers x 72 heads x d 128, fp16): the victim
     is paged decode attention over 16 x 2048 resident tokens (the Fig. 8 decode set,
     P:251) = 72 GiB of KV read per step (64 layer launches) on a HIGH-priority stream; the
@@ -582,10 +582,16 @@ def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:
     dbt = torch.as_tensor(case.dst_bt, device=dev)
     pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
     saved = wk.get_tuning(wk.PATH_INTRA)
-    for cap in (2, 4, 8, 16, 0):
-        wk.set_tuning(wk.PATH_INTRA, **{**saved, "max_ctas": cap})
+    configs = configs or [(f"cap{c or 'none'}", {**saved, "max_ctas": c}) for c in (2, 4, 8, 16, 0)]
+    for name, cfg in configs:
+        wk.set_tuning(wk.PATH_INTRA, **cfg)
         t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, stream=lo_s), 2, 3, lo_s) / 2
-        k = int(math.ceil(n_victim_steps * t_alone * 3.0 / t_mig)) + 2
+        # the victim alone, measured right before this cap's run (removes clock / power drift)
+        torch.cuda.synchronize()
+        ev = victim_run(n_victim_steps)
+        torch.cuda.synchronize()
+        t_ref = float(np.median([ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]))
+        k = int(math.ceil(n_victim_steps * t_ref * 3.0 / t_mig)) + 2
         m0, m1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         torch.cuda.synchronize()
         m0.record(lo_s)
@@ -597,11 +603,12 @@ def run_interference(wk, device, peaks, n_victim_steps=50) -> dict:
         with_mig = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]
         covered = ev[n_victim_steps].elapsed_time(m1) > 0  # migration outlived the victim
         t_with = float(np.median(with_mig))
-        res[f"cap{cap or 'none'}"] = {
+        res[name] = {
             "migration_gbs_alone": round(pb / t_mig / 1e6, 1),
             "migration_hbm_share": round(2 * pb / t_mig / 1e6 / peaks["hbm_gbs"], 4),
+            "victim_ms_alone_adjacent": round(t_ref, 3),
             "victim_ms_with_migration": round(t_with, 3),
-            "slowdown": round(t_with / t_alone - 1.0, 4),
+            "slowdown": round(t_with / t_ref - 1.0, 4),
             "migration_covered_all_victim_steps": bool(covered)}
     wk.set_tuning(wk.PATH_INTRA, **saved)
     del vpool, src, dst

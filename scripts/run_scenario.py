@@ -1,0 +1,29 @@
+"""Run one bench scenario alone on cuda:0 (development helper): python scripts/run_scenario.py <name>"""
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import bench  # noqa: E402
+import paper_conf_isca_fenghzly025_b200 as wk  # noqa: E402
+
+name = sys.argv[1]
+peaks = bench.load_peaks()
+T, S = wk.KERNEL_TMA, wk.KERNEL_SIMT
+small_footprint = [
+    ("tma48kx4_cap4", dict(kernel=T, stage_bytes=49152, stages=4, store_lag=2, ctas_per_sm=1, max_ctas=4)),
+    ("tma16kx4_cap8", dict(kernel=T, stage_bytes=16384, stages=4, store_lag=2, ctas_per_sm=1, max_ctas=8)),
+    ("tma16kx4_cap16", dict(kernel=T, stage_bytes=16384, stages=4, store_lag=2, ctas_per_sm=1, max_ctas=16)),
+    ("tma8kx4_cap16", dict(kernel=T, stage_bytes=8192, stages=4, store_lag=2, ctas_per_sm=1, max_ctas=16)),
+    ("simt32k_cap4", dict(kernel=S, stage_bytes=32768, stages=6, ctas_per_sm=1, max_ctas=4)),
+    ("simt32k_cap8", dict(kernel=S, stage_bytes=32768, stages=6, ctas_per_sm=1, max_ctas=8)),
+    ("tma48kx4_cap4_ef", dict(kernel=T, stage_bytes=49152, stages=4, store_lag=2, ctas_per_sm=1, max_ctas=4,
+                              evict_first=True)),
+]
+fn = {"interference": lambda: bench.run_interference(wk, 0, peaks),
+      "interference_configs": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=30,
+                                                             configs=small_footprint),
+      "pressure": lambda: bench.run_pressure(wk, 0),
+      "stall_free": lambda: bench.run_stall_free(wk, 0),
+      "handoff": lambda: bench.run_handoff(wk, 0)}[name]
+print(json.dumps(fn()))
