@@ -582,27 +582,34 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     dbt = torch.as_tensor(case.dst_bt, device=dev)
     pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
     saved = wk.get_tuning(wk.PATH_INTRA)
-    configs = configs or [(f"cap{c or 'none'}", {**saved, "max_ctas": c}) for c in (2, 4, 8, 16, 0)]
+    configs = configs or (
+        [(f"cap{c or 'none'}", {**saved, "max_ctas": c}) for c in (2, 4, 8, 16, 0)] +
+        [(f"rate{r}GBs", {**saved, "max_ctas": 0, "rate_mbps": r * 1000}) for r in (50, 100, 150, 300)] +
+        [(f"rate{r}GBs_32ctas", {**saved, "max_ctas": 32, "rate_mbps": r * 1000}) for r in (100,)])
+    rounds, n_round = 3, max(10, n_victim_steps // 2)
     for name, cfg in configs:
         wk.set_tuning(wk.PATH_INTRA, **cfg)
         t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, stream=lo_s), 2, 3, lo_s) / 2
-        # the victim alone, measured right before this cap's run (removes clock / power drift)
-        torch.cuda.synchronize()
-        ev = victim_run(n_victim_steps)
-        torch.cuda.synchronize()
-        t_ref = float(np.median([ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]))
-        k = int(math.ceil(n_victim_steps * t_ref * 3.0 / t_mig)) + 2
-        m0, m1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        torch.cuda.synchronize()
-        m0.record(lo_s)
-        for _ in range(k):
-            wk.migrate(src, sbt, dst, dbt, stream=lo_s)
-        m1.record(lo_s)
-        ev = victim_run(n_victim_steps)
-        torch.cuda.synchronize()
-        with_mig = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]
-        covered = ev[n_victim_steps].elapsed_time(m1) > 0  # migration outlived the victim
-        t_with = float(np.median(with_mig))
+        unlimited = cfg.get("max_ctas", 0) == 0 and cfg.get("rate_mbps", 0) == 0
+        alone_all, with_all, covered = [], [], True
+        # `rounds` interleaved pairs (victim alone, then victim + migration): the alone
+        # reference is always adjacent in time (removes clock / power drift)
+        for _ in range(rounds):
+            torch.cuda.synchronize()
+            ev = victim_run(n_round)
+            torch.cuda.synchronize()
+            alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
+            k = int(math.ceil(n_round * float(np.median(alone)) * (3.5 if unlimited else 1.5) / t_mig)) + 1
+            m1 = torch.cuda.Event(enable_timing=True)
+            for _ in range(k):
+                wk.migrate(src, sbt, dst, dbt, stream=lo_s)
+            m1.record(lo_s)
+            ev = victim_run(n_round)
+            torch.cuda.synchronize()
+            with_all += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
+            alone_all += alone
+            covered &= ev[n_round].elapsed_time(m1) > 0  # migration outlived the victim
+        t_ref, t_with = float(np.median(alone_all)), float(np.median(with_all))
         res[name] = {
             "migration_gbs_alone": round(pb / t_mig / 1e6, 1),
             "migration_hbm_share": round(2 * pb / t_mig / 1e6 / peaks["hbm_gbs"], 4),

@@ -265,6 +265,9 @@ typedef struct {
   int32_t max_ctas; /* cap on the grid (e.g. to leave SMs to a decode stream); 0 = none */
   int32_t evict_first; /* 1 = L2 evict-first policy on the copy's loads and stores */
   int32_t store_lag;   /* TMA: stores allowed in flight per CTA (0 = stages / 2) */
+  int32_t rate_mbps;   /* payload rate limit of one op in MB/s (0 = unlimited): bounds the
+                          HBM / link share a migration takes from co-running decode
+                          (S§8(d) interference); paced per CTA with %globaltimer */
 } wind_kv_tuning;
 
 wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t);

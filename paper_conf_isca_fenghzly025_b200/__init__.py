@@ -80,7 +80,7 @@ class MigrateItem(ct.Structure):
 class Tuning(ct.Structure):
     _fields_ = [("kernel", ct.c_int32), ("ctas_per_sm", ct.c_int32), ("stage_bytes", ct.c_int32),
                 ("stages", ct.c_int32), ("max_ctas", ct.c_int32), ("evict_first", ct.c_int32),
-                ("store_lag", ct.c_int32)]
+                ("store_lag", ct.c_int32), ("rate_mbps", ct.c_int32)]
 
 
 _LIB: Optional[ct.CDLL] = None
@@ -389,8 +389,9 @@ def check_device_error(pool: Pool) -> None:
 
 def set_tuning(path: int, kernel: int = KERNEL_AUTO, ctas_per_sm: int = 0, stage_bytes: int = 0,
                stages: int = 0, max_ctas: int = 0, evict_first: bool = False,
-               store_lag: int = 0) -> None:
-    t = Tuning(kernel, ctas_per_sm, stage_bytes, stages, max_ctas, int(evict_first), store_lag)
+               store_lag: int = 0, rate_mbps: int = 0) -> None:
+    t = Tuning(kernel, ctas_per_sm, stage_bytes, stages, max_ctas, int(evict_first), store_lag,
+               rate_mbps)
     _check(lib().wind_kv_set_tuning(path, ct.byref(t)))
 
 

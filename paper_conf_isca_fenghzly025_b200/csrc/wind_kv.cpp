@@ -645,7 +645,14 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   int kernel = t.kernel == kAuto ? (path == WIND_PATH_INTRA ? kTma : kSimt) : t.kernel;
   int64_t grid = static_cast<int64_t>(ctx->sms) * std::max(1, t.ctas_per_sm);
   if (t.max_ctas > 0) grid = std::min<int64_t>(grid, t.max_ctas);
+  // A rate-limited op holds as few SMs as can sustain the rate (one CTA moves ~38 GB/s of
+  // payload intra-device): the SMs a migration occupies cost a co-running HBM-bound decode
+  // kernel more than the bytes it moves (bench c3_interference).
+  if (t.rate_mbps > 0 && t.max_ctas == 0)
+    grid = std::min<int64_t>(grid, std::max<int64_t>(1, (t.rate_mbps + kCtaMBps - 1) / kCtaMBps));
   grid = std::max<int64_t>(1, std::min<int64_t>(grid, p.total_units));
+  // rate limit: each of the `grid` CTAs gets rate / grid; ns per payload byte per CTA
+  p.ns_per_byte = t.rate_mbps > 0 ? static_cast<float>(grid * 1e3 / t.rate_mbps) : 0.f;
   cudaError_t e = launch_copy(p, kernel, static_cast<int>(grid), s);
   if (e != cudaSuccess) return cuda_fail(e, "copy kernel launch");
   g_launches += 1;
@@ -876,7 +883,9 @@ extern "C" wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t)
   n.max_ctas = t->max_ctas;
   n.evict_first = t->evict_first;
   n.store_lag = t->store_lag;
+  n.rate_mbps = t->rate_mbps;
   if (n.store_lag < 0 || n.store_lag >= n.stages) return fail(WIND_ERR_INVALID_ARG, "store_lag out of [0, stages)");
+  if (n.rate_mbps < 0) return fail(WIND_ERR_INVALID_ARG, "rate_mbps < 0");
   if (n.ctas_per_sm < 1 || n.ctas_per_sm > 32) return fail(WIND_ERR_INVALID_ARG, "ctas_per_sm out of [1, 32]");
   if (n.stage_bytes < 16 || n.stage_bytes % 16) return fail(WIND_ERR_INVALID_ARG, "stage_bytes must be a positive multiple of 16");
   if (n.stages < 3 || n.stages > 16) return fail(WIND_ERR_INVALID_ARG, "stages out of [3, 16]");

@@ -15,6 +15,7 @@ namespace wkv {
 // so a slot is reusable as soon as the op that used it has finished.
 constexpr int kCounterSlots = 64;
 constexpr int kMaxSegs = 32;  // segments (runs) per work unit = one warp's table window
+constexpr int kCtaMBps = 30000;  // payload MB/s one copy CTA sustains with headroom (~38 measured)
 
 // One destination of a (possibly batched) migrate launch.
 struct Item {
@@ -49,6 +50,7 @@ struct Params {
   int32_t n_items;
   int32_t evict_first;
   int32_t store_lag;          // TMA consumer: units whose stores may still read smem
+  float ns_per_byte;          // per-CTA pacing (rate limit): 0 = unlimited
   int32_t stages;             // TMA ring depth
   int32_t stage_bytes;        // TMA stage size
   Item items[WIND_KV_MAX_BATCH];

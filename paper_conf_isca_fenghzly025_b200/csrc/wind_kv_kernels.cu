@@ -171,6 +171,31 @@ __device__ __forceinline__ void st_stream_ef(int4* p, const int4& v, uint64_t po
                : "memory");
 }
 
+__device__ __forceinline__ uint64_t globaltimer_ns() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Rate limit (wind_kv_tuning.rate_mbps): a per-CTA pacer.  Before a unit of `bytes` is
+// issued, wait until the CTA's schedule allows it, then push the schedule by
+// bytes * ns_per_byte.  Bursts are bounded: a CTA that fell behind (slow memory) catches up
+// at most one unit ahead of real time.
+struct Pacer {
+  uint64_t next = 0;
+  __device__ __forceinline__ void wait(float ns_per_byte, uint32_t bytes) {
+    if (ns_per_byte <= 0.f) return;
+    uint64_t now = globaltimer_ns();
+    if (next == 0 || next + 20000 < now) next = now;  // start, or behind by > 20 us
+    while (now < next) {
+      const uint64_t d = next - now;
+      __nanosleep(d > 1000000 ? 1000000u : static_cast<unsigned>(d));
+      now = globaltimer_ns();
+    }
+    next += static_cast<uint64_t>(static_cast<float>(bytes) * ns_per_byte);
+  }
+};
+
 // --------------------------------------------------------------------- work decoding
 
 // Decodes unit u into segments (called by a FULL warp; writes segs[] from the lanes that
@@ -320,6 +345,7 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
   if (warp == 0) {  // ------------------------------------------------ producer warp
     const uint64_t pol = ef ? evict_first_policy() : 0;
     const int64_t total = (p.abort_word && *p.abort_word) ? 0 : p.total_units;
+    Pacer pacer;
     int it = 0;
     for (int64_t u = blockIdx.x;; u += gridDim.x, ++it) {
       const int st = it % S;
@@ -335,6 +361,7 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
       __syncwarp();
       if (lane != 0) mbar_arrive(&full[st]);
       if (lane == 0) {
+        pacer.wait(p.ns_per_byte, bytes);
         desc[st].nseg = nseg;
         desc[st].plane = plane;
         mbar_arrive_expect_tx(&full[st], bytes);
@@ -393,12 +420,14 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
   if (blockIdx.x == 0 && tid == 32) publish_untouched_layers(p);  // not the decoding warp
   int32_t cur = p.layer_lo;
   const int64_t total = (p.abort_word && *p.abort_word) ? 0 : p.total_units;
+  Pacer pacer;
   for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
     if (tid < 32) {
       int32_t plane;
       uint32_t bytes;
       const int n = decode_unit(p, u, segs, &plane, &bytes);
       if (tid == 0) {
+        pacer.wait(p.ns_per_byte, bytes);
         s_nseg = n;
         s_plane = plane;
       }

@@ -89,3 +89,36 @@ def test_launch_count_one_kernel_per_op():
     torch.cuda.synchronize()
     assert wk.launch_count() - n0 == 8
     del sh
+
+
+def test_rate_limit_paces_the_copy():
+    """wind_kv_tuning.rate_mbps bounds an op's payload rate (interference budget) without
+    changing its result."""
+    from windgen import SHAPES
+    import windgen.cuda as wg
+    sh = SHAPES["C2"]
+    nb = 300
+    src = wk.Pool(4, sh.n_kv_heads, sh.head_dim, 16, 2, nb)
+    dst = wk.Pool(4, sh.n_kv_heads, sh.head_dim, 16, 2, nb)
+    wg.fill(src.base, src.nbytes, 0, 1, 1)
+    wg.fill(dst.base, dst.nbytes, 0, 1, 2)
+    sbt = torch.randperm(nb, generator=torch.Generator().manual_seed(0))[:256].to(torch.int32).to(DEV)
+    dbt = torch.randperm(nb, generator=torch.Generator().manual_seed(1))[:256].to(torch.int32).to(DEV)
+    payload = 2 * 4 * 256 * sh.chunk_bytes  # 320 MiB
+    saved = wk.get_tuning(wk.PATH_INTRA)
+    s = torch.cuda.Stream(DEV)
+    try:
+        for rate_gbs in (20, 80):
+            wk.set_tuning(wk.PATH_INTRA, **{**saved, "rate_mbps": rate_gbs * 1000})
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(s)
+            wk.migrate(src, sbt, dst, dbt, stream=s)
+            b.record(s)
+            torch.cuda.synchronize()
+            got = payload / (a.elapsed_time(b) * 1e6)
+            assert 0.75 * rate_gbs < got < 1.1 * rate_gbs, (rate_gbs, got)
+    finally:
+        wk.set_tuning(wk.PATH_INTRA, **saved)
+    S = src.tensor().view(4, 2, nb, -1)
+    D = dst.tensor().view(4, 2, nb, -1)
+    assert torch.equal(D[:, :, dbt.long()], S[:, :, sbt.long()])
