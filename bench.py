@@ -319,6 +319,10 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
 
     # (8) C4 memory pressure: evict by swap vs by migration, swap concurrent with hand-off
     out["c4_pressure"] = run_pressure(wk, device)
+    torch.cuda.empty_cache()
+
+    # (9) NEXT-4 policy: Eq. 2 fitted on the decode kernel, theta, trigger, victims
+    out["policy_eq2"] = run_policy_profile(wk, device)
     return out
 
 
@@ -467,6 +471,59 @@ def run_pressure(wk, device, reps: int = 3) -> dict:
                           f"{t_swap / out['evict_by_migration_ms_cap16']:.0f}x faster at an NVLink-rate cap")
     del dpool, host, other, src_inc
     return out
+
+
+def run_policy_profile(wk, device, bw_gbs: float = 550.0) -> dict:
+    """NEXT-4: the Profiler's Eq. 2 (T_decode = a_d * sum(L) + c_d) fitted on the
+    decode-attention kernel over OPT-13B KV (40 layers) at sum(L) = 8K..128K tokens, then the
+    stall-free threshold theta it implies (R6) and the trigger / victim choice for a
+    decode pool at 97 % occupancy (R7, R8)."""
+    import torch
+    import victim
+    from paper_conf_isca_fenghzly025_b200 import policy
+    from windgen import SHAPES, lengths_sharegpt, blocks_for_tokens
+    sh = SHAPES["C2"]
+    dev = torch.device("cuda", device)
+    bs = sh.block_size
+    max_tok = 2048
+    s = torch.cuda.Stream(device)
+    xs, ys = [], []
+    nb = 64 * max_tok // bs
+    pool = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, bs, 2, nb, device=device)
+    pool.tensor().view(torch.float16).normal_()
+    plane = nb * sh.chunk_bytes
+    for B in (4, 8, 16, 32, 64):
+        bt = torch.randperm(nb)[:B * max_tok // bs].to(torch.int32).view(B, -1).to(dev)
+        ctx = torch.full((B,), max_tok, dtype=torch.int32, device=dev)
+        q = torch.randn(B, sh.n_kv_heads, 128, device=dev, dtype=torch.float16)
+        scratch = torch.empty(victim.scratch_floats(B, sh.n_kv_heads, max_tok // bs, 64), device=dev)
+        out = torch.empty(B, sh.n_kv_heads, 128, device=dev)
+
+        def step():
+            for l in range(sh.n_layers):
+                kp = pool.base + 2 * l * plane
+                victim.decode_attention(q, kp, kp + plane, bt, ctx, sh.n_kv_heads, bs, scratch, out,
+                                        blocks_per_split=64, stream=s.cuda_stream)
+        ms = time_device(step, 10, 3, s) / 10
+        xs.append(B * max_tok)
+        ys.append(ms)
+    a, c, r2 = policy.fit_decode_profile(xs, ys)
+    # a decode pool at 97 % occupancy holding 64 ShareGPT-length requests
+    reqb = blocks_for_tokens(lengths_sharegpt(64, 77), bs)
+    n_pool = int(math.ceil(reqb.sum() / 0.97))
+    free = n_pool - int(reqb.sum())
+    trig = policy.should_reschedule(free, n_pool, new_blocks_per_step=len(reqb))
+    need = int(0.05 * n_pool) - free + len(reqb)
+    vic = policy.pick_victims(reqb, need)
+    sum_L = float(reqb.sum() * bs)
+    theta = policy.theta_from_profile(a, c, sum_L, bw_gbs, sh.n_layers, sh.chunk_bytes)
+    del pool
+    return {"eq2_points_sumL_ms": [[int(x), round(y, 3)] for x, y in zip(xs, ys)],
+            "a_d_us_per_token": round(a * 1e3, 5), "c_d_ms": round(c, 4), "r2": round(r2, 5),
+            "pool_blocks": n_pool, "free_blocks": free, "trigger": bool(trig),
+            "victims": vic, "victim_blocks": int(reqb[vic].sum()) if vic else 0,
+            "theta_blocks_at_bw_gbs": {"bw_gbs": bw_gbs, "theta": theta},
+            "note": "decode attention only (Table 1's 4*SUM(L)*H KV read, P:162); GEMMs omitted"}
 
 
 def run_stall_free(wk, device, cap_ctas: int = 16) -> dict:

@@ -24,6 +24,7 @@ fn = {"interference": lambda: bench.run_interference(wk, 0, peaks),
       "interference_configs": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=30,
                                                              configs=small_footprint),
       "pressure": lambda: bench.run_pressure(wk, 0),
+      "policy": lambda: bench.run_policy_profile(wk, 0),
       "stall_free": lambda: bench.run_stall_free(wk, 0),
       "handoff": lambda: bench.run_handoff(wk, 0)}[name]
 print(json.dumps(fn()))
