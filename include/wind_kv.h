@@ -156,8 +156,10 @@ wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind
 
 /* swap_out / swap_in (A6): migrate over all layers of the device pool with a HOST pool as
  * destination / source.  The host pool must cover the device pool's
- * layers.  Executes on the device pool's GPU; SM stores to / loads from mapped pinned
- * memory over PCIe. */
+ * layers.  Executes on the device pool's GPU; SM / TMA stores to and loads from mapped
+ * pinned memory over PCIe.  A host pool's layer flags live in mapped host memory and are
+ * updated without PCIe atomics, so ops INTO one host pool must not overlap in time (ops on
+ * one stream never do); the host observes swap_out progress by reading the flags. */
 wind_status wind_kv_swap_out(const wind_kv_pool* dev, const int32_t* dev_bt,
                              wind_kv_pool* host, const int32_t* host_bt, int32_t n_blocks,
                              void* stream);
