@@ -122,3 +122,17 @@ def test_rate_limit_paces_the_copy():
     S = src.tensor().view(4, 2, nb, -1)
     D = dst.tensor().view(4, 2, nb, -1)
     assert torch.equal(D[:, :, dbt.long()], S[:, :, sbt.long()])
+
+
+def test_plain_c_abi_user():
+    """examples/c_abi_example.c drives the library through the C ABI alone."""
+    import os
+    import subprocess
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    exe = os.path.join(root, "examples", "c_abi_example")
+    if not os.path.exists(exe):
+        import __graft_entry__
+        __graft_entry__.build_c_example()
+    out = subprocess.run([exe], capture_output=True, text=True, timeout=300)
+    assert out.returncode == 0, out.stderr
+    assert "c_abi_example OK" in out.stdout
