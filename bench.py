@@ -821,7 +821,23 @@ def run_gpu(args) -> None:
     n_movers = parallel.movers(world)
     total_bytes = pb * n_movers
     a2a = None
+    peer_alt = None
     if world > 1 and args.scenarios:
+        # the peer-path kernel choice was not measurable on one GPU in round 1: time the
+        # alternatives on the real link (same op, 3 steps each, max over ranks)
+        peer_alt = {}
+        saved = wk.get_tuning(wk.PATH_PEER)
+        for name, cfg in [("simt_96ctas", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=32768,
+                                                max_ctas=96)),
+                          ("simt_4x148", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768)),
+                          ("tma_148", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4,
+                                           store_lag=2)),
+                          ("tma_32", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4,
+                                          store_lag=2, max_ctas=32))]:
+            wk.set_tuning(wk.PATH_PEER, **cfg)
+            ms_alt, = parallel.max_over_ranks([time_device(step, 3, 3, stream, barrier) / 3])
+            peer_alt[name] = round(pb / ms_alt / 1e6, 1)
+        wk.set_tuning(wk.PATH_PEER, **saved)
         del src, dst
         torch.cuda.empty_cache()
         a2a = run_all_to_all(wk, rank, world, local, peaks, scale=args.a2a_scale)
@@ -844,7 +860,7 @@ def run_gpu(args) -> None:
                     "per_launch_bytes": pb}
         extra["roofline"] = roof
         if a2a is not None:
-            extra["scenarios"] = {"c5_all_to_all": a2a}
+            extra["scenarios"] = {"c5_all_to_all": a2a, "peer_kernel_gbs_per_pair": peer_alt}
         if world == 1 and not args.no_cpu_baseline:
             # the cpu_baseline leg: the oracle timed on the host cores, and (outside every
             # timed region) the oracle's sampled check of this run's GPU output
