@@ -815,7 +815,8 @@ def run_gpu(args) -> None:
         dst.read_flags(flags_host, stream=stream)  # the step's result: layer_done[] D2H
         stream.synchronize()
 
-    ms_e2e_local = time_device(e2e_step, max(3, args.steps // 2), 2, stream, barrier) / max(3, args.steps // 2)
+    e2e_steps = max(3, args.steps // 2)
+    ms_e2e_local = time_device(e2e_step, e2e_steps, args.warmup, stream, barrier) / e2e_steps
 
     ms_step, ms_e2e = parallel.max_over_ranks([ms_step_local, ms_e2e_local])
     n_movers = parallel.movers(world)
