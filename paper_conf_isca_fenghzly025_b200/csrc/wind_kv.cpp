@@ -480,18 +480,24 @@ wind_status route(const wind_kv_pool* src, const wind_kv_pool* dst, int* exec, i
   }
   const bool same_gpu = memcmp(src->uuid, dst->uuid, 16) == 0;
   *path = same_gpu ? WIND_PATH_INTRA : WIND_PATH_PEER;
-  if (!src->imported && !dst->imported && src->desc.device != dst->desc.device) {
+  if (src->imported && dst->imported)
+    return fail(WIND_ERR_UNSUPPORTED, "at least one pool must be local to this process");
+  // an imported pool is mapped for the device it was imported into: the op must run there
+  const wind_kv_pool* imp = src->imported ? src : (dst->imported ? dst : nullptr);
+  if (imp && imp->desc.device != *exec)
+    return fail(WIND_ERR_INVALID_ARG, "imported pool is mapped for device %d but the op executes on %d",
+                imp->desc.device, *exec);
+  // a local pool on another device of this process: enable peer access from the executing one
+  const wind_kv_pool* other = (src->desc.device != *exec) ? src : dst;
+  if (!other->imported && other->desc.device != *exec) {
     int can = 0;
-    cudaDeviceCanAccessPeer(&can, src->desc.device, dst->desc.device);
-    if (!can) return fail(WIND_ERR_NO_PEER, "device %d cannot access device %d", src->desc.device,
-                          dst->desc.device);
-    DeviceGuard g(src->desc.device);
-    cudaError_t e = cudaDeviceEnablePeerAccess(dst->desc.device, 0);  // once per pair
+    cudaDeviceCanAccessPeer(&can, *exec, other->desc.device);
+    if (!can) return fail(WIND_ERR_NO_PEER, "device %d cannot access device %d", *exec, other->desc.device);
+    DeviceGuard g(*exec);
+    cudaError_t e = cudaDeviceEnablePeerAccess(other->desc.device, 0);  // once per pair
     if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_fail(e, "cudaDeviceEnablePeerAccess");
     cudaGetLastError();
   }
-  if (src->imported && dst->imported)
-    return fail(WIND_ERR_UNSUPPORTED, "at least one pool must be local to this process");
   return WIND_OK;
 }
 
