@@ -612,17 +612,24 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             victim.decode_attention(q, kp, kp + plane, bt, ctx, sh.n_kv_heads, bs, scratch, out,
                                     blocks_per_split=bps, stream=hi_s.cuda_stream)
 
-    def victim_run(n):
-        ev = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
-        ev[0].record(hi_s)
-        for i in range(n):
-            victim_step()
-            ev[i + 1].record(hi_s)
-        return ev
-
     for _ in range(5):
         victim_step()
     torch.cuda.synchronize()
+    # a decode step is one CUDA-graph replay (as serving engines run it): its 128 launches
+    # cannot be delayed by host-side contention with the thread that enqueues migrations
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph, stream=hi_s):
+        victim_step()
+    torch.cuda.synchronize()
+
+    def victim_run(n):
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
+        with torch.cuda.stream(hi_s):
+            ev[0].record(hi_s)
+            for i in range(n):
+                graph.replay()
+                ev[i + 1].record(hi_s)
+        return ev
     ev = victim_run(n_victim_steps)
     torch.cuda.synchronize()
     alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]
@@ -635,37 +642,58 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     case = migration_case("C3")
     src = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
     dst = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag)
-    sbt = torch.as_tensor(case.src_bt, device=dev)
-    dbt = torch.as_tensor(case.dst_bt, device=dev)
+    d_tabs = (torch.as_tensor(case.src_bt, device=dev), torch.as_tensor(case.dst_bt, device=dev))
+    h_tabs = (torch.as_tensor(case.src_bt).pin_memory(), torch.as_tensor(case.dst_bt).pin_memory())
     pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
     saved = wk.get_tuning(wk.PATH_INTRA)
     configs = configs or (
+        [("control_no_migration", {**saved, "null_feeder": True})] +
         [(f"cap{c or 'none'}", {**saved, "max_ctas": c}) for c in (2, 4, 8, 16, 0)] +
         [(f"rate{r}GBs", {**saved, "max_ctas": 0, "rate_mbps": r * 1000}) for r in (50, 100, 150, 300)] +
-        [(f"rate{r}GBs_32ctas", {**saved, "max_ctas": 32, "rate_mbps": r * 1000}) for r in (100,)])
+        [(f"rate{r}GBs_32ctas", {**saved, "max_ctas": 32, "rate_mbps": r * 1000}) for r in (100,)] +
+        [(f"copy_engines_rate{r}GBs", {**saved, "kernel": wk.KERNEL_COPY_ENGINE, "rate_mbps": r * 1000})
+         for r in (50, 100, 150, 300)])
     rounds, n_round = 3, max(10, n_victim_steps // 2)
     for name, cfg in configs:
+        cfg = dict(cfg)
+        null = cfg.pop("null_feeder", False)  # control: the feeder thread runs, moves nothing
         wk.set_tuning(wk.PATH_INTRA, **cfg)
-        t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, stream=lo_s), 2, 3, lo_s) / 2
-        unlimited = cfg.get("max_ctas", 0) == 0 and cfg.get("rate_mbps", 0) == 0
+        ce = cfg.get("kernel") == wk.KERNEL_COPY_ENGINE
+        sbt, dbt = (h_tabs[0].data_ptr(), h_tabs[1].data_ptr()) if ce else d_tabs
+        t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, n=case.n, stream=lo_s), 2, 3, lo_s) / 2
         alone_all, with_all, covered = [], [], True
         # `rounds` interleaved pairs (victim alone, then victim + migration): the alone
-        # reference is always adjacent in time (removes clock / power drift)
+        # reference is always adjacent in time (removes clock / power drift).  A feeder
+        # thread keeps exactly one migration op in flight on the low-priority stream for the
+        # whole victim run (the victim's launches are never queued behind migration work on
+        # the host; ctypes releases the GIL inside the library calls).
         for _ in range(rounds):
             torch.cuda.synchronize()
             ev = victim_run(n_round)
             torch.cuda.synchronize()
             alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
-            k = int(math.ceil(n_round * float(np.median(alone)) * (3.5 if unlimited else 1.5) / t_mig)) + 1
-            m1 = torch.cuda.Event(enable_timing=True)
-            for _ in range(k):
-                wk.migrate(src, sbt, dst, dbt, stream=lo_s)
-            m1.record(lo_s)
+            stop, started, n_ops = threading.Event(), threading.Event(), [0]
+
+            def feeder():
+                while not stop.is_set():
+                    if null:
+                        started.set()
+                        time.sleep(0.001)
+                        continue
+                    wk.migrate(src, sbt, dst, dbt, n=case.n, stream=lo_s)
+                    started.set()
+                    lo_s.synchronize()
+                    n_ops[0] += 1
+            th = threading.Thread(target=feeder, daemon=True)
+            th.start()
+            started.wait()
             ev = victim_run(n_round)
             torch.cuda.synchronize()
+            stop.set()
+            th.join()
+            covered &= th is not None and n_ops[0] >= 1
             with_all += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
             alone_all += alone
-            covered &= ev[n_round].elapsed_time(m1) > 0  # migration outlived the victim
         t_ref, t_with = float(np.median(alone_all)), float(np.median(with_all))
         res[name] = {
             "migration_gbs_alone": round(pb / t_mig / 1e6, 1),

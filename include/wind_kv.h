@@ -255,7 +255,11 @@ wind_status wind_kv_check_device_error(const wind_kv_pool* pool);
 /* ------------------------------------------------------------------ tuning & misc */
 
 /* Kernel selection and launch shape, per path.  Defaults are the measured best on B200
- * (DESIGN.md §Kernels).  kernel: 0 = auto, 1 = TMA bulk staged copy, 2 = SIMT 16-B
+ * (DESIGN.md §Kernels).  kernel: 3 = copy engines (DMA, zero SMs: the low-interference
+ * background mode; needs host-readable block tables; one cudaMemcpy2DAsync per run of
+ * adjacent blocks; flags published once after all layers; rate_mbps paces it with
+ * 1-thread sleep kernels between copies),
+ * 0 = auto, 1 = TMA bulk staged copy, 2 = SIMT 16-B
  * vector copy.  ctas_per_sm, stage_bytes (TMA stage / SIMT unit bytes, multiple of 16),
  * stages (TMA ring depth); 0 keeps the current value. */
 typedef enum { WIND_PATH_INTRA = 0, WIND_PATH_PEER = 1, WIND_PATH_HOST = 2 } wind_path;

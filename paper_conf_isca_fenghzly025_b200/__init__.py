@@ -37,7 +37,7 @@ OK = 0
 LOC_DEVICE, LOC_HOST = 0, 1
 POOL_DEBUG = 0x1
 PATH_INTRA, PATH_PEER, PATH_HOST = 0, 1, 2
-KERNEL_AUTO, KERNEL_TMA, KERNEL_SIMT = 0, 1, 2
+KERNEL_AUTO, KERNEL_TMA, KERNEL_SIMT, KERNEL_COPY_ENGINE = 0, 1, 2, 3
 IPC_HANDLE_BYTES = 512
 MAX_BATCH = 16
 
@@ -322,10 +322,13 @@ def migrate_heads(src: Pool, src_bt, dst: Pool, dst_bt, src_head_lo: int, dst_he
 
 def migrate_batch(src: Pool, items: Sequence[tuple], layer_lo: int, layer_hi: int,
                   stream=None) -> None:
-    """wind_kv_migrate_batch: items = [(dst_pool, src_bt, dst_bt), ...] in one launch."""
+    """wind_kv_migrate_batch: items = [(dst_pool, src_bt, dst_bt[, n]), ...] in one launch
+    (n is required when the tables are passed as raw addresses)."""
     arr = (MigrateItem * len(items))()
-    for k, (dst, sbt, dbt) in enumerate(items):
-        arr[k] = MigrateItem(dst.handle, _ptr(sbt), _ptr(dbt), _len(sbt))
+    for k, item in enumerate(items):
+        dst, sbt, dbt = item[:3]
+        n = item[3] if len(item) > 3 else _len(sbt)
+        arr[k] = MigrateItem(dst.handle, _ptr(sbt), _ptr(dbt), n)
     dev = src.device if not src.is_host else items[0][0].device
     _check(lib().wind_kv_migrate_batch(src.handle, arr, len(items), layer_lo, layer_hi,
                                        _stream(stream, dev)))

@@ -547,6 +547,71 @@ wind_status debug_check(DevCtx* ctx, int exec, const wind_kv_pool* src, const Op
   return WIND_OK;
 }
 
+bool host_readable(const void* ptr) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, ptr) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeHost || a.type == cudaMemoryTypeUnregistered ||
+         a.type == cudaMemoryTypeManaged;
+}
+
+// Copy-engine path (tuning kernel = 3): the DMA engines move the bytes, no SM is used, so a
+// co-running decode kernel keeps every SM (bench c3_interference).  One cudaMemcpy2DAsync
+// per run of adjacent blocks covers all planes (rows = the 2 (hi - lo) planes, row pitch =
+// each pool's plane stride).  The tables must be host-readable (the driver needs every
+// address at enqueue time); the layer flags are published by one tiny kernel afterwards
+// (stream order: after every copy), so per-layer streaming is not available on this path.
+wind_status copy_engine_op(const Params& p, const OpItem* items, int n_items, cudaStream_t s,
+                           int32_t rate_mbps) {
+  const size_t rows = static_cast<size_t>(2) * p.n_layers;
+  // rate limit: a pace kernel stamps the op start; after copies worth >= 20 us of the
+  // budget, a pace kernel holds the stream until start + bytes_so_far / rate.  The stamp
+  // lives in this op's (otherwise unused) arrival-counter slot.
+  unsigned long long* t0 = reinterpret_cast<unsigned long long*>(p.counters + WIND_KV_MAX_LAYERS - 2);
+  double sched_ns = 0, last_paced = 0;
+  int launches = 0;
+  if (rate_mbps > 0) {
+    WKV_CUDA(launch_pace(t0, 0, 1, s), "pace kernel launch");
+    ++launches;
+  }
+  for (int j = 0; j < n_items; ++j) {
+    const OpItem& it = items[j];
+    if (it.n == 0) continue;
+    if (!host_readable(it.sbt) || !host_readable(it.dbt))
+      return fail(WIND_ERR_UNSUPPORTED, "copy-engine path needs host-readable block tables");
+    const Item& q = p.items[j];
+    const bool co = q.coalesce != 0;
+    for (int32_t i = 0; i < it.n;) {
+      int32_t k = 1;
+      while (co && i + k < it.n && it.sbt[i + k] == it.sbt[i] + k && it.dbt[i + k] == it.dbt[i] + k) ++k;
+      const uint8_t* sp = p.src_plane0 + static_cast<int64_t>(it.sbt[i]) * p.s_chunk;
+      uint8_t* dp = q.dst_plane0 + static_cast<int64_t>(it.dbt[i]) * q.d_chunk;
+      WKV_CUDA(cudaMemcpy2DAsync(dp, static_cast<size_t>(q.d_plane_stride), sp,
+                                 static_cast<size_t>(p.s_plane_stride), static_cast<size_t>(p.copy) * k, rows,
+                                 cudaMemcpyDefault, s),
+               "cudaMemcpy2DAsync");
+      if (rate_mbps > 0) {
+        sched_ns += static_cast<double>(p.copy) * k * rows * 1e3 / rate_mbps;
+        if (sched_ns - last_paced >= 20000) {
+          WKV_CUDA(launch_pace(t0, static_cast<uint64_t>(sched_ns), 0, s), "pace kernel launch");
+          last_paced = sched_ns;
+          ++launches;
+        }
+      }
+      i += k;
+    }
+  }
+  if (rate_mbps > 0 && sched_ns > last_paced) {
+    WKV_CUDA(launch_pace(t0, static_cast<uint64_t>(sched_ns), 0, s), "pace kernel launch");
+    ++launches;
+  }
+  WKV_CUDA(launch_flag_bump(p, s), "flag kernel launch");
+  g_launches += 1 + launches;
+  return WIND_OK;
+}
+
 // The common op: src -> items[] over layers [lo, hi) on `stream`.
 wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
                    int32_t hi, void* stream, const HeadRange& hr = HeadRange()) {
@@ -649,6 +714,11 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   p.abort_word = debug ? ctx->err : nullptr;
 
   int kernel = t.kernel == kAuto ? (path == WIND_PATH_INTRA ? kTma : kSimt) : t.kernel;
+  if (kernel == kCopyEngine) {
+    if ((st = copy_engine_op(p, items, n_items, s, t.rate_mbps)) != WIND_OK) return st;
+    for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
+    return WIND_OK;
+  }
   int64_t grid = static_cast<int64_t>(ctx->sms) * std::max(1, t.ctas_per_sm);
   if (t.max_ctas > 0) grid = std::min<int64_t>(grid, t.max_ctas);
   // A rate-limited op holds as few SMs as can sustain the rate (one CTA moves ~38 GB/s of
@@ -881,7 +951,7 @@ extern "C" wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t)
   if (path < 0 || path > 2 || !t) return fail(WIND_ERR_INVALID_ARG, "bad path or NULL tuning");
   std::lock_guard<std::mutex> lk(g_tune_mu);
   wind_kv_tuning n = g_tune[path];
-  if (t->kernel < 0 || t->kernel > 2) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0, 1 or 2");
+  if (t->kernel < 0 || t->kernel > 3) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0, 1, 2 or 3");
   n.kernel = t->kernel;
   if (t->ctas_per_sm) n.ctas_per_sm = t->ctas_per_sm;
   if (t->stage_bytes) n.stage_bytes = t->stage_bytes;

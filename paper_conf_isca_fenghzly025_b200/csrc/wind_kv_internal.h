@@ -56,7 +56,14 @@ struct Params {
   Item items[WIND_KV_MAX_BATCH];
 };
 
-enum Kernel { kAuto = 0, kTma = 1, kSimt = 2 };
+enum Kernel { kAuto = 0, kTma = 1, kSimt = 2, kCopyEngine = 3 };
+
+// Copy-engine path: after the DMA copies of an op (stream-ordered), one tiny kernel adds 1
+// to every layer flag of every item (release, system scope).
+cudaError_t launch_flag_bump(const Params& p, cudaStream_t s);
+// Copy-engine rate limit: a 1-thread kernel; `first` stamps the op start in *t0, later
+// launches sleep until *t0 + target_ns.
+cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s);
 
 // Launchers (wind_kv_kernels.cu).  Return cudaGetLastError() after the launch.
 cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s);

@@ -467,6 +467,35 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
   if (tid == 0) arrive_layers(p, cur, p.layer_lo + p.n_layers);
 }
 
+// ------------------------------------------------- copy-engine path: flag publication
+
+__global__ void flag_bump_kernel(const __grid_constant__ Params p) {
+  // the DMA copies before this kernel in stream order have completed; make that ordering
+  // visible system-wide before the flags move
+  fence_sys();
+  for (int j = 0; j < p.n_items; ++j)
+    for (int f = threadIdx.x; f < p.items[j].d_layers; f += blockDim.x)
+      bump_flag(p.items[j].flags + f, p.items[j].host_flags);
+}
+
+// Copy-engine pacing: one thread (no SM resources worth mentioning, so a rate-limited DMA
+// migration stays off the SMs).  The first launch of an op stamps the op's start time in
+// *t0; every later launch sleeps until t0 + target_ns (the schedule of the bytes copied
+// so far), so command overheads are absorbed and the average rate is exact.
+__global__ void pace_kernel(unsigned long long* t0, uint64_t target_ns, int first) {
+  if (first) {
+    *t0 = globaltimer_ns();
+    return;
+  }
+  const uint64_t until = *reinterpret_cast<volatile unsigned long long*>(t0) + target_ns;
+  uint64_t now = globaltimer_ns();
+  while (now < until) {
+    const uint64_t d = until - now;
+    __nanosleep(d > 1000000 ? 1000000u : static_cast<unsigned>(d));
+    now = globaltimer_ns();
+  }
+}
+
 // -------------------------------------------------------- debug-pool device table check
 
 __global__ void table_count_kernel(const int32_t* sbt, const int32_t* dbt, int32_t n,
@@ -513,6 +542,16 @@ cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s) {
   } else {
     simt_copy_kernel<<<grid, kSimtThreads, 0, s>>>(p);
   }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s) {
+  pace_kernel<<<1, 1, 0, s>>>(t0, target_ns, first);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_flag_bump(const Params& p, cudaStream_t s) {
+  flag_bump_kernel<<<1, 128, 0, s>>>(p);
   return cudaGetLastError();
 }
 

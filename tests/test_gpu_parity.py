@@ -287,3 +287,26 @@ def test_batch_migrate_matches_sequential_oracle():
         assert O.migrate(s0, geom(src), sb, want, geom(d), db, 0, 3) == O.OK
         np.testing.assert_array_equal(read(d), want)
         assert d.layer_ticket() == 1 and [d.layer_count(l) for l in range(3)] == [1, 1, 1]
+
+
+@pytest.mark.parametrize("variant", ["shuffled", "sequential"])
+def test_copy_engine_path_matches_oracle(variant):
+    """kernel = 3 (DMA engines, zero SMs): same result as the oracle; host-readable tables
+    required; flags published once per op."""
+    wk.set_tuning(wk.PATH_INTRA, kernel=wk.KERNEL_COPY_ENGINE)
+    case = migration_case("C1", variant=variant, scale=0.5)
+    sh = case.shape
+    src, s0 = make_pool(sh, case.nb_src, 21)
+    dst, d0 = make_pool(sh, case.nb_dst, 22)
+    want = d0.copy()
+    assert O.migrate(s0, geom(src), case.src_bt, want, geom(dst), case.dst_bt, 2, 10) == O.OK
+    hs = torch.as_tensor(case.src_bt).pin_memory()
+    hd = torch.as_tensor(case.dst_bt).pin_memory()
+    n0 = wk.launch_count()
+    wk.migrate(src, hs.data_ptr(), dst, hd.data_ptr(), n=case.n, layer_lo=2, layer_hi=10)
+    np.testing.assert_array_equal(read(dst), want)
+    assert wk.launch_count() - n0 == 1  # the flag kernel only
+    assert [dst.layer_count(l) for l in range(sh.n_layers)] == [1] * sh.n_layers
+    with pytest.raises(wk.WindKVError) as e:  # device tables: not readable by the host
+        wk.migrate(src, tab(case.src_bt), dst, tab(case.dst_bt))
+    assert e.value.status == -10
