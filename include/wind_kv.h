@@ -277,6 +277,14 @@ typedef struct {
 } wind_kv_tuning;
 
 wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t);
+
+/* wind_kv_migrate with a per-op tuning override (NULL = the path's current tuning): e.g.
+ * the early stages of a stall-free migration on the copy engines with a rate budget and
+ * its final stage on the TMA kernel at full rate.  Every field of the override is taken
+ * literally (no "0 keeps" rule) and validated like set_tuning; kernel 0 = auto. */
+wind_status wind_kv_migrate_ex(const wind_kv_pool* src, const int32_t* src_bt, wind_kv_pool* dst,
+                               const int32_t* dst_bt, int32_t n_blocks, int32_t layer_lo,
+                               int32_t layer_hi, const wind_kv_tuning* tuning, void* stream);
 wind_status wind_kv_get_tuning(int32_t path, wind_kv_tuning* t);
 
 /* Number of kernels this process has launched through the library (all ops). */

@@ -49,7 +49,8 @@ EXPORTED_SYMBOLS = [
     "wind_kv_layer_ticket",
     "wind_kv_layer_wait", "wind_kv_layer_count", "wind_kv_read_flags", "wind_kv_validate", "wind_kv_plan_compact",
     "wind_kv_plan_rebalance", "wind_kv_check_device_error", "wind_kv_set_tuning",
-    "wind_kv_get_tuning", "wind_kv_launch_count", "wind_kv_status_string", "wind_kv_last_error",
+    "wind_kv_get_tuning", "wind_kv_migrate_ex", "wind_kv_launch_count", "wind_kv_status_string",
+    "wind_kv_last_error",
     "wind_kv_version",
 ]
 
@@ -118,6 +119,7 @@ def lib() -> ct.CDLL:
         "wind_kv_check_device_error": [P],
         "wind_kv_set_tuning": [I32, ct.POINTER(Tuning)],
         "wind_kv_get_tuning": [I32, ct.POINTER(Tuning)],
+        "wind_kv_migrate_ex": [P, P, P, P, I32, I32, I32, ct.POINTER(Tuning), P],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -305,6 +307,24 @@ def migrate(src: Pool, src_bt, dst: Pool, dst_bt, n: Optional[int] = None,
     hi = min(src.layers[1], dst.layers[1]) if layer_hi is None else layer_hi
     _check(lib().wind_kv_migrate(src.handle, _ptr(src_bt), dst.handle, _ptr(dst_bt), n, lo, hi,
                                  _stream(stream, _exec_device(src, dst))))
+
+
+def tuning(kernel: int = KERNEL_TMA, ctas_per_sm: int = 1, stage_bytes: int = 49152, stages: int = 4,
+           max_ctas: int = 0, evict_first: bool = False, store_lag: int = 2, rate_mbps: int = 0) -> Tuning:
+    """A complete per-op tuning (every field explicit) for migrate_ex."""
+    return Tuning(kernel, ctas_per_sm, stage_bytes, stages, max_ctas, int(evict_first), store_lag, rate_mbps)
+
+
+def migrate_ex(src: Pool, src_bt, dst: Pool, dst_bt, tuning_override: Optional[Tuning],
+               n: Optional[int] = None, layer_lo: Optional[int] = None, layer_hi: Optional[int] = None,
+               stream=None) -> None:
+    """wind_kv_migrate_ex: migrate with a per-op tuning (None = the path's current one)."""
+    n = _len(src_bt) if n is None else n
+    lo = max(src.layers[0], dst.layers[0]) if layer_lo is None else layer_lo
+    hi = min(src.layers[1], dst.layers[1]) if layer_hi is None else layer_hi
+    tp = ct.byref(tuning_override) if tuning_override is not None else None
+    _check(lib().wind_kv_migrate_ex(src.handle, _ptr(src_bt), dst.handle, _ptr(dst_bt), n, lo, hi, tp,
+                                    _stream(stream, _exec_device(src, dst))))
 
 
 def migrate_heads(src: Pool, src_bt, dst: Pool, dst_bt, src_head_lo: int, dst_head_lo: int,

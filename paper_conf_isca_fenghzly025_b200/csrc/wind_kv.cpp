@@ -614,7 +614,8 @@ wind_status copy_engine_op(const Params& p, const OpItem* items, int n_items, cu
 
 // The common op: src -> items[] over layers [lo, hi) on `stream`.
 wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
-                   int32_t hi, void* stream, const HeadRange& hr = HeadRange()) {
+                   int32_t hi, void* stream, const HeadRange& hr = HeadRange(),
+                   const wind_kv_tuning* override_tuning = nullptr) {
   if (!src) return fail(WIND_ERR_INVALID_ARG, "src pool is NULL");
   if (n_items < 1 || n_items > WIND_KV_MAX_BATCH) return fail(WIND_ERR_INVALID_ARG, "n_items out of range");
   int exec = -1, path = 0;
@@ -640,7 +641,9 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   DevCtx* ctx;
   if ((st = dev_ctx(exec, &ctx)) != WIND_OK) return st;
   wind_kv_tuning t;
-  {
+  if (override_tuning) {
+    t = *override_tuning;  // validated by wind_kv_migrate_ex
+  } else {
     std::lock_guard<std::mutex> lk(g_tune_mu);
     t = g_tune[path];
   }
@@ -969,6 +972,24 @@ extern "C" wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t)
     return fail(WIND_ERR_INVALID_ARG, "stages * stage_bytes exceeds shared memory");
   g_tune[path] = n;
   return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_migrate_ex(const wind_kv_pool* src, const int32_t* src_bt,
+                                          wind_kv_pool* dst, const int32_t* dst_bt, int32_t n_blocks,
+                                          int32_t layer_lo, int32_t layer_hi, const wind_kv_tuning* tuning,
+                                          void* stream) {
+  if (!dst) return fail(WIND_ERR_INVALID_ARG, "dst pool is NULL");
+  if (tuning) {  // validate the override like set_tuning would, then apply it to this op only
+    if (tuning->kernel < 0 || tuning->kernel > 3) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0..3");
+    if (tuning->ctas_per_sm < 1 || tuning->ctas_per_sm > 32 || tuning->stage_bytes < 16 ||
+        tuning->stage_bytes % 16 || tuning->stages < 3 || tuning->stages > 16 || tuning->store_lag < 0 ||
+        tuning->store_lag >= tuning->stages || tuning->rate_mbps < 0 || tuning->max_ctas < 0)
+      return fail(WIND_ERR_INVALID_ARG, "override tuning out of range (all fields explicit, see wind_kv.h)");
+    if (tuning->kernel != kSimt && tma_smem_bytes(tuning->stages, tuning->stage_bytes) > 227 * 1024)
+      return fail(WIND_ERR_INVALID_ARG, "stages * stage_bytes exceeds shared memory");
+  }
+  OpItem it{dst, src_bt, dst_bt, n_blocks};
+  return run_op(src, &it, 1, layer_lo, layer_hi, stream, HeadRange(), tuning);
 }
 
 extern "C" wind_status wind_kv_get_tuning(int32_t path, wind_kv_tuning* t) {

@@ -532,8 +532,22 @@ size_t tma_smem_bytes(int stages, int stage_bytes) {
 
 cudaError_t prepare_kernels(int device, size_t max_tma_smem) {
   (void)device;
-  return cudaFuncSetAttribute(tma_copy_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                              static_cast<int>(max_tma_smem));
+  cudaError_t e = cudaFuncSetAttribute(tma_copy_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                       static_cast<int>(max_tma_smem));
+  if (e != cudaSuccess) return e;
+  // Load every kernel now (pool creation): with CUDA's lazy module loading the first launch
+  // of a kernel loads its code, which synchronises the whole device — an op must never do
+  // that on the hot path.
+  const void* fns[] = {reinterpret_cast<const void*>(simt_copy_kernel),
+                       reinterpret_cast<const void*>(flag_bump_kernel),
+                       reinterpret_cast<const void*>(pace_kernel),
+                       reinterpret_cast<const void*>(table_count_kernel),
+                       reinterpret_cast<const void*>(table_judge_kernel)};
+  for (const void* f : fns) {
+    cudaFuncAttributes a;
+    if ((e = cudaFuncGetAttributes(&a, f)) != cudaSuccess) return e;
+  }
+  return cudaSuccess;
 }
 
 cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s) {

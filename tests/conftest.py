@@ -1,7 +1,11 @@
 import os
 import sys
 
-import pytest
+# More hardware work queues than the default 8, so streams never share one (a paced
+# copy-engine migration holds its queue while it sleeps; see include/wind_kv.h tuning).
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
+
+import pytest  # noqa: E402
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 for _p in (ROOT, os.path.join(ROOT, "tests")):
