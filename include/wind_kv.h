@@ -258,7 +258,10 @@ wind_status wind_kv_check_device_error(const wind_kv_pool* pool);
  * (DESIGN.md §Kernels).  kernel: 3 = copy engines (DMA, zero SMs: the low-interference
  * background mode; needs host-readable block tables; one cudaMemcpy2DAsync per run of
  * adjacent blocks; flags published once after all layers; rate_mbps paces it with
- * 1-thread sleep kernels between copies),
+ * 1-thread sleep kernels between copies — those hold the stream's hardware queue, so work
+ * of another stream that CUDA maps onto the same queue waits behind them: raise
+ * CUDA_DEVICE_MAX_CONNECTIONS (e.g. 32) and keep few streams; the TMA / SIMT kernels pace
+ * inside the kernel and never hold a queue),
  * 0 = auto, 1 = TMA bulk staged copy, 2 = SIMT 16-B
  * vector copy.  ctas_per_sm, stage_bytes (TMA stage / SIMT unit bytes, multiple of 16),
  * stages (TMA ring depth); 0 keeps the current value. */
