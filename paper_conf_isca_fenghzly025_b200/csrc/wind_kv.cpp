@@ -17,6 +17,8 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: ranges show up in ncu / nsys, free otherwise
+
 #include "wind_kv_internal.h"
 
 using namespace wkv;
@@ -618,6 +620,10 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
                    const wind_kv_tuning* override_tuning = nullptr) {
   if (!src) return fail(WIND_ERR_INVALID_ARG, "src pool is NULL");
   if (n_items < 1 || n_items > WIND_KV_MAX_BATCH) return fail(WIND_ERR_INVALID_ARG, "n_items out of range");
+  struct NvtxRange {  // one NVTX range per op (the enqueue, on the host timeline)
+    NvtxRange() { nvtxRangePushA("wind_kv op"); }
+    ~NvtxRange() { nvtxRangePop(); }
+  } nvtx_range;
   int exec = -1, path = 0;
   wind_status st;
   for (int j = 0; j < n_items; ++j) {
