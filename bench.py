@@ -915,6 +915,12 @@ def run_gpu(args) -> None:
                     "h2d_bytes_per_step": int(8 * case.n), "d2h_bytes_per_step": int(4 * sh.n_layers)},
             "gpu_launches": int(launches),
             "clocks": clk.summary(),
+            # the paper's only migration number, as context (A800, not a target): one
+            # 2048-token OPT-13B request = 1.5625 GiB, "~65 ms" over PCIe Gen4 x16
+            "paper_context": {
+                "p120_request_gib": 1.5625, "p120_pcie_gen4_ms": 65.0, "p120_implied_gbs": 25.8,
+                "same_request_ms_at_this_rate": round(1.5625 * GiB / (value / n_movers * 1e6), 3),
+                "same_request_ms_at_nvlink5_770gbs": round(1.5625 * GiB / 770e6, 3)},
             **extra,
         }
         print(json.dumps(line), flush=True)
