@@ -708,6 +708,11 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     q.d_flag_lo = lo - d->desc.first_layer;
     q.d_layers = d->desc.n_layers;
     q.host_flags = d->desc.loc == WIND_LOC_HOST;
+    // GPU-scope publication only when both pools live on the executing GPU (same physical
+    // device: every reader of the data and of the flags goes through this GPU's L2)
+    q.sys_scope = !(src->desc.loc == WIND_LOC_DEVICE && d->desc.loc == WIND_LOC_DEVICE &&
+                    memcmp(src->uuid, d->uuid, 16) == 0);
+    p.sys_scope |= q.sys_scope;
     const int64_t u = p.parts > 1 ? static_cast<int64_t>(it.n) * p.parts
                                   : (static_cast<int64_t>(it.n) + p.group - 1) / p.group;
     if (u + base_units > INT32_MAX) return fail(WIND_ERR_UNSUPPORTED, "too many work units");

@@ -32,6 +32,9 @@ struct Item {
   int32_t units;           // work units per (layer, kv) plane for this item
   int32_t unit_base;       // prefix of `units` over previous items
   int32_t host_flags;      // flags live in mapped host memory: bump by plain RMW, not red.sys
+  int32_t sys_scope;       // data or flags leave this GPU (peer / host pool): publish with
+                           // system-scope fences; else GPU scope (a .sys fence costs ~1 us
+                           // and stalls the copy stream, S DESIGN §6 publication cost)
 };
 
 struct Params {
@@ -53,6 +56,7 @@ struct Params {
   float ns_per_byte;          // per-CTA pacing (rate limit): 0 = unlimited
   int32_t stages;             // TMA ring depth
   int32_t stage_bytes;        // TMA stage size
+  int32_t sys_scope;          // any item has sys_scope
   Item items[WIND_KV_MAX_BATCH];
 };
 

@@ -135,6 +135,10 @@ __device__ __forceinline__ void fence_sys() {
   asm volatile("fence.acq_rel.sys;" ::: "memory");
 }
 
+__device__ __forceinline__ void fence_gpu() {
+  asm volatile("fence.acq_rel.gpu;" ::: "memory");
+}
+
 __device__ __forceinline__ void fence_async_global() {
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
@@ -254,13 +258,17 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
   return __popc(heads);
 }
 
-// Adds 1 to a layer flag with release semantics at system scope.  Device-memory flags
-// (local or peer) use a red.release.sys reduction; flags of a host pool (mapped pinned
-// memory, where PCIe may not carry atomics) use a volatile RMW + release store — the
-// executing device is then the only writer (wind_kv.h: one op at a time per host pool).
-__device__ __forceinline__ void bump_flag(uint32_t* f, bool host) {
-  if (!host) {
-    red_release_sys_add(f, 1u);
+// Adds 1 to a layer flag with release semantics.  Device-memory flags use a red.release
+// reduction, at system scope when the item's data or flags leave this GPU (peer pool) and
+// at GPU scope otherwise; flags of a host pool (mapped pinned memory, where PCIe may not
+// carry atomics) use a volatile RMW + release.sys store — the executing device is then the
+// only writer (wind_kv.h: one op at a time per host pool).
+__device__ __forceinline__ void bump_flag(uint32_t* f, const Item& it) {
+  if (!it.host_flags) {
+    if (it.sys_scope)
+      red_release_sys_add(f, 1u);
+    else
+      asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(f) : "memory");
   } else {
     const uint32_t v = *reinterpret_cast<volatile uint32_t*>(f);
     asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(v + 1u) : "memory");
@@ -301,19 +309,49 @@ __device__ __forceinline__ void bulk_wait_read_n(int n) {
   }
 }
 
+// Same, but full completion (the stores' writes performed, not only their smem reads).
+__device__ __forceinline__ void bulk_wait_done_n(int n) {
+  switch (n) {
+    case 0: asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); break;
+    case 1: asm volatile("cp.async.bulk.wait_group 1;" ::: "memory"); break;
+    case 2: asm volatile("cp.async.bulk.wait_group 2;" ::: "memory"); break;
+    case 3: asm volatile("cp.async.bulk.wait_group 3;" ::: "memory"); break;
+    case 4: asm volatile("cp.async.bulk.wait_group 4;" ::: "memory"); break;
+    case 5: asm volatile("cp.async.bulk.wait_group 5;" ::: "memory"); break;
+    case 6: asm volatile("cp.async.bulk.wait_group 6;" ::: "memory"); break;
+    default: asm volatile("cp.async.bulk.wait_group 7;" ::: "memory"); break;
+  }
+}
+
 // Arrive on layers [from, to) (global ids) of this op; the last CTA publishes.  Caller has
-// made this CTA's stores of those layers complete and ordered before this call.
+// made this CTA's stores of those layers complete and ordered before this call.  The
+// counter atomics of a range are issued 8 at a time (independent round trips in flight).
+// Scope: when data and flags stay on this GPU (p.sys_scope == 0) every observer — the
+// consumer stream's wait, the kernels it releases, another process's CTAs on this device —
+// reads through this GPU's L2, so GPU-scope fences suffice; a fence.acq_rel.sys costs
+// ~1 us and, issued per layer, cost a 32-layer op ~50 us.
 __device__ void arrive_layers(const Params& p, int32_t from, int32_t to) {
   if (from >= to) return;
-  fence_sys();
-  for (int32_t l = from; l < to; ++l) {
-    uint32_t* c = p.counters + (l - p.layer_lo);
-    const uint32_t old = atomicAdd(c, 1u);
-    if (old == gridDim.x - 1) {
-      fence_sys();
+  if (p.sys_scope)
+    fence_sys();
+  else
+    fence_gpu();
+  for (int32_t l0 = from; l0 < to; l0 += 8) {
+    uint32_t old[8];
+#pragma unroll
+    for (int k = 0; k < 8; ++k)
+      if (l0 + k < to) old[k] = atomicAdd(p.counters + (l0 + k - p.layer_lo), 1u);
+#pragma unroll
+    for (int k = 0; k < 8; ++k) {
+      const int32_t l = l0 + k;
+      if (l >= to || old[k] != gridDim.x - 1) continue;
+      if (p.sys_scope)
+        fence_sys();
+      else
+        fence_gpu();
       for (int j = 0; j < p.n_items; ++j)
-        bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (l - p.layer_lo), p.items[j].host_flags);
-      *reinterpret_cast<volatile uint32_t*>(c) = 0u;  // slot reusable by a later op
+        bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (l - p.layer_lo), p.items[j]);
+      *reinterpret_cast<volatile uint32_t*>(p.counters + (l - p.layer_lo)) = 0u;  // slot reusable
     }
   }
 }
@@ -378,18 +416,30 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
     // stores allowed to be still reading their stage: half the ring (the other half is
     // the producer's load lookahead)
     const int lag = p.store_lag > 0 ? p.store_lag : (S / 2 > 0 ? S / 2 : 1);
+    // Layer arrivals without draining the store pipeline: when unit `it` opens a later
+    // layer, the stores of layers [cur, layer) are the bulk groups < it.  The arrival is
+    // deferred until `lag` newer groups have been committed; then a full wait_group<lag>
+    // (instead of this iteration's .read wait) makes exactly those groups complete.  A
+    // second boundary while one is pending (< lag units per layer) resolves the first one
+    // on the spot with a shallower wait.
     int32_t cur = p.layer_lo;  // layers < cur have been arrived on by this CTA
+    int32_t pend_to = -1;      // pending arrival on [cur, pend_to) once groups < pend_it are done
+    int pend_it = 0;
     for (int it = 0;; ++it) {
       const int st = it % S;
       mbar_wait(&full[st], (it / S) & 1);
       const int nseg = desc[st].nseg;
       if (nseg < 0) break;
       const int32_t layer = p.layer_lo + desc[st].plane / 2;
-      if (layer > cur) {  // this CTA is done with layers [cur, layer)
-        bulk_wait_all();
-        fence_async_global();
-        arrive_layers(p, cur, layer);
-        cur = layer;
+      if (layer > (pend_to >= 0 ? pend_to : cur)) {  // this CTA is done with layers < layer
+        if (pend_to >= 0) {
+          bulk_wait_done_n(it - pend_it);  // the it - pend_it groups >= pend_it may stay pending
+          fence_async_global();
+          arrive_layers(p, cur, pend_to);
+          cur = pend_to;
+        }
+        pend_to = layer;
+        pend_it = it;
       }
       const uint8_t* sbuf = buf + static_cast<size_t>(st) * SB;
       for (int k = 0; k < nseg; ++k) {
@@ -397,7 +447,15 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
         bulk_store(g.dst, sbuf + g.soff, g.len, ef, pol);
       }
       bulk_commit();
-      bulk_wait_read_n(lag);  // stores of units <= it - lag have read their stage
+      if (pend_to >= 0 && it - pend_it + 1 >= lag) {
+        bulk_wait_done_n(it - pend_it + 1);  // groups < pend_it complete (and <= it - lag read)
+        fence_async_global();
+        arrive_layers(p, cur, pend_to);
+        cur = pend_to;
+        pend_to = -1;
+      } else {
+        bulk_wait_read_n(lag);  // stores of units <= it - lag have read their stage
+      }
       if (it >= lag) mbar_arrive(&empty[(it - lag) % S]);
     }
     bulk_wait_all();
@@ -475,7 +533,7 @@ __global__ void flag_bump_kernel(const __grid_constant__ Params p) {
   fence_sys();
   for (int j = 0; j < p.n_items; ++j)
     for (int f = threadIdx.x; f < p.items[j].d_layers; f += blockDim.x)
-      bump_flag(p.items[j].flags + f, p.items[j].host_flags);
+      bump_flag(p.items[j].flags + f, p.items[j]);
 }
 
 // Copy-engine pacing: one thread (no SM resources worth mentioning, so a rate-limited DMA

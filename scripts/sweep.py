@@ -17,8 +17,9 @@ import paper_conf_isca_fenghzly025_b200 as wk  # noqa: E402
 import windgen.cuda as wg  # noqa: E402
 from windgen import migration_case, SHAPES, KVShape  # noqa: E402
 
-PEAK = json.load(open(os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))),
-                                   "MEASURED_PEAKS.json")))["hbm_gbs"]
+import bench  # noqa: E402
+
+PEAK = bench.load_peaks()["hbm_gbs"]
 dev = torch.device("cuda", 0)
 
 
