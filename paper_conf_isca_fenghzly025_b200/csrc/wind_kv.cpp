@@ -133,7 +133,9 @@ wind_kv_tuning g_tune[3] = {
     // threads keep ~3 MiB of stores in flight (> 2 us x 900 GB/s) and leave SMs to the
     // co-running prefill / decode.  Not yet tuned on a multi-GPU box (one GPU per round-1 call).
     /* PEER  */ {kSimt, 1, 32768, 6, 96, 0, 0},
-    /* HOST  */ {kTma, 1, 49152, 4, 64, 0, 2},  // PCIe-bound: 64 SMs reach the link rate
+    // HOST: PCIe-bound; 8 CTAs reach the same 52 / 51 GB/s as 64 or 148 (sweep r01: SM
+    // stores to pinned memory plateau at 0.91 of the copy engines' 57 / 55.5 GB/s)
+    /* HOST  */ {kTma, 1, 49152, 4, 8, 0, 2},
 };
 
 }  // namespace

@@ -143,10 +143,6 @@ __device__ __forceinline__ void fence_async_global() {
   asm volatile("fence.proxy.async.global;" ::: "memory");
 }
 
-__device__ __forceinline__ void red_release_sys_add(uint32_t* p, uint32_t v) {
-  asm volatile("red.release.sys.global.add.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
 __device__ __forceinline__ int4 ld_stream(const int4* p) {
   int4 r;
   asm volatile("ld.global.nc.L1::no_allocate.v4.s32 {%0, %1, %2, %3}, [%4];"
@@ -258,20 +254,20 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
   return __popc(heads);
 }
 
-// Adds 1 to a layer flag with release semantics.  Device-memory flags use a red.release
-// reduction, at system scope when the item's data or flags leave this GPU (peer pool) and
-// at GPU scope otherwise; flags of a host pool (mapped pinned memory, where PCIe may not
-// carry atomics) use a volatile RMW + release.sys store — the executing device is then the
+// Adds 1 to a layer flag.  The caller has issued the release fence (fence.acq_rel at
+// system scope when the item's data or flags leave this GPU, at GPU scope otherwise), so the
+// increment itself is relaxed: one fence publishes every flag a thread bumps after it.
+// Device-memory flags use a red reduction; flags of a host pool (mapped pinned memory, where
+// PCIe may not carry atomics) a volatile read-modify-write — the executing device is then the
 // only writer (wind_kv.h: one op at a time per host pool).
 __device__ __forceinline__ void bump_flag(uint32_t* f, const Item& it) {
-  if (!it.host_flags) {
-    if (it.sys_scope)
-      red_release_sys_add(f, 1u);
-    else
-      asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(f) : "memory");
-  } else {
+  if (it.host_flags) {
     const uint32_t v = *reinterpret_cast<volatile uint32_t*>(f);
-    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(f), "r"(v + 1u) : "memory");
+    asm volatile("st.relaxed.sys.global.u32 [%0], %1;" ::"l"(f), "r"(v + 1u) : "memory");
+  } else if (it.sys_scope) {
+    asm volatile("red.relaxed.sys.global.add.u32 [%0], 1;" ::"l"(f) : "memory");
+  } else {
+    asm volatile("red.relaxed.gpu.global.add.u32 [%0], 1;" ::"l"(f) : "memory");
   }
 }
 
@@ -341,14 +337,17 @@ __device__ void arrive_layers(const Params& p, int32_t from, int32_t to) {
 #pragma unroll
     for (int k = 0; k < 8; ++k)
       if (l0 + k < to) old[k] = atomicAdd(p.counters + (l0 + k - p.layer_lo), 1u);
+    uint32_t last = 0;  // layers of this batch whose last arrival is this CTA's
 #pragma unroll
-    for (int k = 0; k < 8; ++k) {
-      const int32_t l = l0 + k;
-      if (l >= to || old[k] != gridDim.x - 1) continue;
-      if (p.sys_scope)
-        fence_sys();
-      else
-        fence_gpu();
+    for (int k = 0; k < 8; ++k)
+      if (l0 + k < to && old[k] == gridDim.x - 1) last |= 1u << k;
+    if (!last) continue;
+    if (p.sys_scope)  // one release fence for every flag published below
+      fence_sys();
+    else
+      fence_gpu();
+    for (uint32_t m = last; m; m &= m - 1) {
+      const int32_t l = l0 + __ffs(m) - 1;
       for (int j = 0; j < p.n_items; ++j)
         bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (l - p.layer_lo), p.items[j]);
       *reinterpret_cast<volatile uint32_t*>(p.counters + (l - p.layer_lo)) = 0u;  // slot reusable

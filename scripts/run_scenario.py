@@ -19,6 +19,12 @@ small_footprint = [
     ("simt32k_cap8", dict(kernel=S, stage_bytes=32768, stages=6, ctas_per_sm=1, max_ctas=8)),
     ("tma48kx4_cap4_ef", dict(kernel=T, stage_bytes=49152, stages=4, store_lag=2, ctas_per_sm=1, max_ctas=4,
                               evict_first=True)),
+    ("tma48kx4_cap2", dict(kernel=T, stage_bytes=49152, stages=4, store_lag=2, ctas_per_sm=1, max_ctas=2)),
+    ("tma16kx3_cap2", dict(kernel=T, stage_bytes=16384, stages=3, store_lag=1, ctas_per_sm=1, max_ctas=2)),
+    ("tma16kx3_rate50", dict(kernel=T, stage_bytes=16384, stages=3, store_lag=1, ctas_per_sm=1, max_ctas=0,
+                             rate_mbps=50000)),
+    ("simt32k_rate50", dict(kernel=S, stage_bytes=32768, stages=4, ctas_per_sm=1, max_ctas=2, rate_mbps=50000)),
+    ("ce_rate50", dict(kernel=3, stage_bytes=49152, stages=4, rate_mbps=50000)),
 ]
 fn = {"interference": lambda: bench.run_interference(wk, 0, peaks),
       "interference_configs": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=30,

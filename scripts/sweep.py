@@ -51,6 +51,7 @@ def host_sweep():
                         nblk, loc="host")
         bt = torch.randperm(nblk + 10)[:nblk].to(torch.int32).to(dev)
         hbt = torch.arange(nblk, dtype=torch.int32, device=dev)
+        bt_h, hbt_h = bt.cpu().pin_memory(), hbt.cpu().pin_memory()
         pb = 2 * sh.n_layers * nblk * sh.chunk_bytes
         for cfg in [dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768),
                     dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=2, stage_bytes=32768),
@@ -60,10 +61,19 @@ def host_sweep():
                     dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=32768, stages=6),
                     dict(kernel=wk.KERNEL_TMA, ctas_per_sm=2, stage_bytes=16384, stages=6),
                     dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768, max_ctas=64),
-                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, max_ctas=64)]:
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, max_ctas=64),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, max_ctas=32),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, max_ctas=16),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, max_ctas=8),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, max_ctas=4),
+                    dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=32768, stages=6, max_ctas=8),
+                    dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=65536, max_ctas=8),
+                    dict(kernel=wk.KERNEL_COPY_ENGINE, stage_bytes=49152, stages=4)]:
             wk.set_tuning(wk.PATH_HOST, **cfg)
-            mo = timeit(lambda: wk.swap_out(dpool, bt, hpool, hbt, stream=s), s, reps=5)
-            mi = timeit(lambda: wk.swap_in(hpool, hbt, dpool, bt, stream=s), s, reps=5)
+            ce = cfg["kernel"] == wk.KERNEL_COPY_ENGINE
+            a, b = (bt_h, hbt_h) if ce else (bt, hbt)
+            mo = timeit(lambda: wk.swap_out(dpool, a, hpool, b, n=nblk, stream=s), s, reps=5)
+            mi = timeit(lambda: wk.swap_in(hpool, b, dpool, a, n=nblk, stream=s), s, reps=5)
             print(json.dumps(dict(case=name, mode="host", **cfg, out_gbs=round(pb / mo / 1e6, 2),
                                   in_gbs=round(pb / mi / 1e6, 2))), flush=True)
         hb = torch.empty(pb, dtype=torch.uint8, pin_memory=True)
