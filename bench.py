@@ -121,25 +121,29 @@ def make_pool(wk, shape, nb, device, seed, tag, loc="device"):
     return p
 
 
-def time_device(fn, steps: int, warmup: int, stream, barrier=None):
+def time_device(fn, steps: int, warmup: int, stream, barrier=None, per_step=None):
     """W untimed warm-up steps, then EXACTLY `steps` steps between CUDA events on `stream`,
-    barrier + synchronize on both sides.  Returns total ms."""
+    barrier + synchronize on both sides.  Returns total ms.  With a list `per_step`, an
+    event is also recorded between steps and the per-step ms are appended to it."""
     import torch
     for _ in range(warmup):
         fn()
     torch.cuda.synchronize()
     if barrier:
         barrier()
-    e0 = torch.cuda.Event(enable_timing=True)
-    e1 = torch.cuda.Event(enable_timing=True)
-    e0.record(stream)
-    for _ in range(steps):
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(steps + 1 if per_step is not None else 2)]
+    ev[0].record(stream)
+    for i in range(steps):
         fn()
-    e1.record(stream)
+        if per_step is not None:
+            ev[i + 1].record(stream)
+    ev[-1].record(stream)
     torch.cuda.synchronize()
     if barrier:
         barrier()
-    return e0.elapsed_time(e1)
+    if per_step is not None:
+        per_step += [ev[i].elapsed_time(ev[i + 1]) for i in range(steps)]
+    return ev[0].elapsed_time(ev[-1])
 
 
 # ------------------------------------------------------------------ cpu baseline
@@ -794,7 +798,10 @@ def run_gpu(args) -> None:
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("gloo", rank=rank, world_size=world)
+        import datetime
+        # bounded: a rank that fails in a scenario must not hang the others forever
+        dist.init_process_group("gloo", rank=rank, world_size=world,
+                                timeout=datetime.timedelta(seconds=600))
     barrier = (lambda: dist.barrier()) if world > 1 else None
     peaks = load_peaks()
 
@@ -823,8 +830,9 @@ def run_gpu(args) -> None:
 
     torch.cuda.synchronize()
     launches0 = wk.launch_count()
+    step_ms: list = []
     with ClockSampler(local) as clk:
-        ms_total = time_device(step, args.steps, args.warmup, stream, barrier)
+        ms_total = time_device(step, args.steps, args.warmup, stream, barrier, per_step=step_ms)
     launches = wk.launch_count() - launches0 - (args.warmup if role != "decode" else 0)
     ms_step_local = ms_total / args.steps
     # e2e: tables from pinned host memory H2D, the migrate, the layer flags read back D2H
@@ -851,25 +859,33 @@ def run_gpu(args) -> None:
     total_bytes = pb * n_movers
     a2a = None
     peer_alt = None
+    scen_error = None
     if world > 1 and args.scenarios:
-        # the peer-path kernel choice was not measurable on one GPU in round 1: time the
-        # alternatives on the real link (same op, 3 steps each, max over ranks)
-        peer_alt = {}
-        saved = wk.get_tuning(wk.PATH_PEER)
-        for name, cfg in [("simt_96ctas", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=32768,
-                                                max_ctas=96)),
-                          ("simt_4x148", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768)),
-                          ("tma_148", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4,
-                                           store_lag=2)),
-                          ("tma_32", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4,
-                                          store_lag=2, max_ctas=32))]:
-            wk.set_tuning(wk.PATH_PEER, **cfg)
-            ms_alt, = parallel.max_over_ranks([time_device(step, 3, 3, stream, barrier) / 3])
-            peer_alt[name] = round(pb / ms_alt / 1e6, 1)
-        wk.set_tuning(wk.PATH_PEER, **saved)
-        del src, dst
-        torch.cuda.empty_cache()
-        a2a = run_all_to_all(wk, rank, world, local, peaks, scale=args.a2a_scale)
+        # The multi-GPU scenarios never ran on more than one GPU in round 1 (one GPU per
+        # gpurun call): a failure there is reported in the line, never loses the headline.
+        try:
+            # the peer-path kernel choice: time the alternatives on the real link (same op,
+            # 3 steps each, max over ranks)
+            peer_alt = {}
+            saved = wk.get_tuning(wk.PATH_PEER)
+            for name, cfg in [("simt_96ctas", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=32768,
+                                                    max_ctas=96)),
+                              ("simt_4x148", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768)),
+                              ("tma_148", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4,
+                                               store_lag=2)),
+                              ("tma_32", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4,
+                                              store_lag=2, max_ctas=32))]:
+                wk.set_tuning(wk.PATH_PEER, **cfg)
+                ms_alt, = parallel.max_over_ranks([time_device(step, 3, 3, stream, barrier) / 3])
+                peer_alt[name] = round(pb / ms_alt / 1e6, 1)
+            wk.set_tuning(wk.PATH_PEER, **saved)
+            torch.cuda.synchronize()
+            del src, dst
+            torch.cuda.empty_cache()
+            a2a = run_all_to_all(wk, rank, world, local, peaks, scale=args.a2a_scale)
+        except Exception as e:  # noqa: BLE001 — reported, not swallowed
+            scen_error = f"{type(e).__name__}: {e}"[:400]
+            print(f"[bench rank {rank}] multi-GPU scenario failed: {scen_error}", file=sys.stderr, flush=True)
     value = total_bytes / ms_step / 1e6  # GB/s
     e2e_value = total_bytes / ms_e2e / 1e6
 
@@ -888,8 +904,10 @@ def run_gpu(args) -> None:
                     "frac": round(kernel_gbs / 900.0, 4), "traffic": None, "peak_src": "nominal",
                     "per_launch_bytes": pb}
         extra["roofline"] = roof
-        if a2a is not None:
+        if a2a is not None or scen_error is not None:
             extra["scenarios"] = {"c5_all_to_all": a2a, "peer_kernel_gbs_per_pair": peer_alt}
+            if scen_error is not None:
+                extra["scenarios"]["error"] = scen_error
         if world == 1 and not args.no_cpu_baseline:
             # the cpu_baseline leg: the oracle timed on the host cores, and (outside every
             # timed region) the oracle's sampled check of this run's GPU output
@@ -914,6 +932,9 @@ def run_gpu(args) -> None:
             "e2e": {"value": round(e2e_value, 2), "unit": "GB/s",
                     "h2d_bytes_per_step": int(8 * case.n), "d2h_bytes_per_step": int(4 * sh.n_layers)},
             "gpu_launches": int(launches),
+            "step_ms_rank0": {"p10": round(float(np.percentile(step_ms, 10)), 4),
+                              "p50": round(float(np.percentile(step_ms, 50)), 4),
+                              "p90": round(float(np.percentile(step_ms, 90)), 4)},
             "clocks": clk.summary(),
             # the paper's only migration number, as context (A800, not a target): one
             # 2048-token OPT-13B request = 1.5625 GiB, "~65 ms" over PCIe Gen4 x16
