@@ -327,6 +327,61 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
 
     # (9) NEXT-4 policy: Eq. 2 fitted on the decode kernel, theta, trigger, victims
     out["policy_eq2"] = run_policy_profile(wk, device)
+    torch.cuda.empty_cache()
+
+    # (10) NEXT-3 backups (read-once fan-out) and TP reshard (head-range migrate)
+    out["next3_backup_reshard"] = run_next3(wk, device, peaks)
+    torch.cuda.empty_cache()
+    return out
+
+
+def run_next3(wk, device, peaks, steps=10, warmup=3) -> dict:
+    """NEXT-3 (P:233 backups; P:128 / Table 3 mismatched TP placements), C2 geometry at half
+    size (1452 blocks, 17.7 GiB):
+    * backup fan-out: the same blocks into TWO destination pools.  read_once = one launch
+      whose items share one source table (the TMA kernel stages each unit once and stores it
+      twice: 3 x payload of DRAM traffic); per_item = one launch, separate table objects
+      (each item re-reads the source: 4 x payload); two_launches = two migrates.
+    * TP-2 -> TP-1 reshard: two half-head (20 of 40 heads) source pools pushed into one
+      full pool at head offsets 0 and 20 (wind_kv_migrate_heads, 80 KiB spans)."""
+    import torch
+    from windgen import migration_case, KVShape, SHAPES
+    sh = SHAPES["C2"]
+    dev = torch.device("cuda", device)
+    s = torch.cuda.Stream(device)
+    hbm = peaks["hbm_gbs"]
+    case = migration_case("C2", scale=0.5)
+    src = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
+    a = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag)
+    b = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag + 1)
+    sbt = torch.as_tensor(case.src_bt, device=dev)
+    sbt2 = sbt.clone()
+    dbt = torch.as_tensor(case.dst_bt, device=dev)
+    pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
+    out = {"blocks": case.n, "payload_gib_per_destination": round(pb / GiB, 2)}
+    runs = {"read_once": lambda: wk.migrate_batch(src, [(a, sbt, dbt), (b, sbt, dbt)], 0, sh.n_layers, stream=s),
+            "per_item": lambda: wk.migrate_batch(src, [(a, sbt, dbt), (b, sbt2, dbt)], 0, sh.n_layers, stream=s),
+            "two_launches": lambda: (wk.migrate(src, sbt, a, dbt, stream=s), wk.migrate(src, sbt, b, dbt, stream=s))}
+    for name, fn in runs.items():
+        ms = time_device(fn, steps, warmup, s) / steps
+        dram = (3 if name == "read_once" else 4) * pb
+        out[f"fanout2_{name}"] = {"ms": round(ms, 3), "delivered_gbs": round(2 * pb / ms / 1e6, 1),
+                                  "dram_gbs": round(dram / ms / 1e6, 1),
+                                  "hbm_frac": round(dram / ms / 1e6 / hbm, 3)}
+    del src, a, b
+    torch.cuda.empty_cache()
+    half = KVShape("OPT-13B TP-2 shard", sh.n_layers, sh.n_kv_heads // 2, sh.head_dim, sh.elem_bytes)
+    shards = [make_pool(wk, half, case.nb_src, device, case.content_seed, 40 + r) for r in range(2)]
+    full = make_pool(wk, sh, case.nb_dst, device, case.content_seed, 50)
+
+    def reshard():
+        for r, sp in enumerate(shards):
+            wk.migrate_heads(sp, sbt, full, dbt, 0, r * half.n_kv_heads, half.n_kv_heads, stream=s)
+    ms = time_device(reshard, steps, warmup, s) / steps
+    out["tp2_to_tp1_reshard"] = {"ms": round(ms, 3), "gbs": round(pb / ms / 1e6, 1),
+                                 "hbm_frac": round(2 * pb / ms / 1e6 / hbm, 3),
+                                 "span_kib": half.n_kv_heads * sh.block_size * sh.head_dim * sh.elem_bytes // 1024}
+    del shards, full
     return out
 
 

@@ -199,7 +199,11 @@ typedef struct {
 
 /* Batched migrate (A8): items[0..n_items) all read from `src`, layers [lo, hi), in one
  * launch on `stream`.  Destination pools must be pairwise distinct objects with
- * disjoint memory (the planner guarantees it).  n_items <= WIND_KV_MAX_BATCH. */
+ * disjoint memory (the planner guarantees it).  n_items <= WIND_KV_MAX_BATCH.
+ * Read-once fan-out (KV backups): when 2-4 items pass the SAME src_bt
+ * pointer with the same n_blocks and the op runs on the TMA kernel, each source unit is
+ * staged once and stored to every destination (DRAM traffic (1 + k) x payload instead of
+ * 2k x); results are identical to the per-item path. */
 wind_status wind_kv_migrate_batch(const wind_kv_pool* src, const wind_kv_migrate_item* items,
                                   int32_t n_items, int32_t layer_lo, int32_t layer_hi,
                                   void* stream);

@@ -15,6 +15,7 @@ namespace wkv {
 // so a slot is reusable as soon as the op that used it has finished.
 constexpr int kCounterSlots = 64;
 constexpr int kMaxSegs = 32;  // segments (runs) per work unit = one warp's table window
+constexpr int kMaxFan = 4;    // destinations of a read-once fan-out (TMA kernel)
 constexpr int kCtaMBps = 30000;  // payload MB/s one copy CTA sustains with headroom (~38 measured)
 
 // One destination of a (possibly batched) migrate launch.
@@ -57,6 +58,9 @@ struct Params {
   int32_t stages;             // TMA ring depth
   int32_t stage_bytes;        // TMA stage size
   int32_t sys_scope;          // any item has sys_scope
+  int32_t fan;                // > 1: read-once fan-out — every item shares items[0]'s source
+                              // table and units; each staged unit is stored to all `fan`
+                              // destinations (TMA kernel only; 1 otherwise)
   Item items[WIND_KV_MAX_BATCH];
 };
 

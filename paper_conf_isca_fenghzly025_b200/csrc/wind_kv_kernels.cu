@@ -52,6 +52,7 @@ struct __align__(16) Desc {
   int32_t nseg;   // -1 = end of work
   int32_t plane;  // (l - lo) * 2 + kv
   Seg segs[kMaxSegs];
+  uint8_t* fdst[kMaxFan - 1][kMaxSegs];  // fan-out: segment k's address in destination 1 + f
 };
 
 // ----------------------------------------------------------------------- PTX helpers
@@ -200,13 +201,19 @@ struct Pacer {
 
 // Decodes unit u into segments (called by a FULL warp; writes segs[] from the lanes that
 // own a segment).  Returns the (warp-uniform) segment count; *plane_out, *bytes_out.
+// Fan-out (p.fan > 1, fdst != nullptr): the units walk items[0]'s source table; a run must
+// be adjacent in the source and in EVERY destination, and fdst[f][k] receives segment k's
+// address in destination 1 + f.
 __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs,
-                                           int32_t* plane_out, uint32_t* bytes_out) {
+                                           uint8_t* (*fdst)[kMaxSegs], int32_t* plane_out,
+                                           uint32_t* bytes_out) {
   const int lane = threadIdx.x & 31;
   const int64_t plane = u / p.units_per_plane;
   int32_t r = static_cast<int32_t>(u - plane * p.units_per_plane);
   int j = 0;
-  while (j + 1 < p.n_items && r >= p.items[j + 1].unit_base) ++j;
+  if (p.fan <= 1)
+    while (j + 1 < p.n_items && r >= p.items[j + 1].unit_base) ++j;
+  const int fan = fdst ? p.fan : 1;
   const Item& it = p.items[j];
   r -= it.unit_base;
   const uint8_t* splane = p.src_plane0 + plane * p.s_plane_stride;
@@ -226,6 +233,10 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
       segs[0].len = len;
       segs[0].soff = 0;
     }
+    if (lane > 0 && lane < fan) {  // lane f: destination f of the fan-out
+      const Item& fi = p.items[lane];
+      fdst[lane - 1][0] = fi.dst_plane0 + plane * fi.d_plane_stride + fi.dbt[i] * fi.d_chunk + off;
+    }
     *bytes_out = len;
     return 1;
   }
@@ -233,13 +244,25 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
   const int32_t i0 = r * p.group;
   const int cnt = min(p.group, it.n - i0);
   int32_t s = 0, d = 0;
+  int32_t df[kMaxFan - 1] = {0, 0, 0};
   if (lane < cnt) {
     s = it.sbt[i0 + lane];
     d = it.dbt[i0 + lane];
+#pragma unroll
+    for (int f = 1; f < kMaxFan; ++f)
+      if (f < fan) df[f - 1] = p.items[f].dbt[i0 + lane];
   }
   const int32_t ps = __shfl_up_sync(kFull, s, 1);
   const int32_t pd = __shfl_up_sync(kFull, d, 1);
-  const bool head = lane < cnt && (lane == 0 || !(it.coalesce && s == ps + 1 && d == pd + 1));
+  bool adj = it.coalesce && s == ps + 1 && d == pd + 1;
+#pragma unroll
+  for (int f = 1; f < kMaxFan; ++f) {
+    if (f < fan) {  // fan is warp-uniform
+      const int32_t pf = __shfl_up_sync(kFull, df[f - 1], 1);
+      adj = adj && df[f - 1] == pf + 1;
+    }
+  }
+  const bool head = lane < cnt && (lane == 0 || !adj);
   const uint32_t heads = __ballot_sync(kFull, head);
   if (head) {
     const int k = __popc(heads & ((1u << lane) - 1u));       // prefix popcount
@@ -249,6 +272,13 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
     segs[k].dst = dplane + d * CD;
     segs[k].len = static_cast<uint32_t>((end - lane) * CP);
     segs[k].soff = static_cast<uint32_t>(lane * CP);
+#pragma unroll
+    for (int f = 1; f < kMaxFan; ++f) {
+      if (f < fan) {
+        const Item& fi = p.items[f];
+        fdst[f - 1][k] = fi.dst_plane0 + plane * fi.d_plane_stride + df[f - 1] * fi.d_chunk;
+      }
+    }
   }
   *bytes_out = static_cast<uint32_t>(cnt * CP);
   return __popc(heads);
@@ -394,7 +424,7 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
       }
       int32_t plane;
       uint32_t bytes;
-      const int nseg = decode_unit(p, u, desc[st].segs, &plane, &bytes);
+      const int nseg = decode_unit(p, u, desc[st].segs, desc[st].fdst, &plane, &bytes);
       __syncwarp();
       if (lane != 0) mbar_arrive(&full[st]);
       if (lane == 0) {
@@ -445,6 +475,11 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
         const Seg& g = desc[st].segs[k];
         bulk_store(g.dst, sbuf + g.soff, g.len, ef, pol);
       }
+      for (int f = 1; f < p.fan; ++f)  // read-once fan-out: the same staged bytes again
+        for (int k = 0; k < nseg; ++k) {
+          const Seg& g = desc[st].segs[k];
+          bulk_store(desc[st].fdst[f - 1][k], sbuf + g.soff, g.len, ef, pol);
+        }
       bulk_commit();
       if (pend_to >= 0 && it - pend_it + 1 >= lag) {
         bulk_wait_done_n(it - pend_it + 1);  // groups < pend_it complete (and <= it - lag read)
@@ -482,7 +517,7 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
     if (tid < 32) {
       int32_t plane;
       uint32_t bytes;
-      const int n = decode_unit(p, u, segs, &plane, &bytes);
+      const int n = decode_unit(p, u, segs, nullptr, &plane, &bytes);
       if (tid == 0) {
         pacer.wait(p.ns_per_byte, bytes);
         s_nseg = n;

@@ -32,5 +32,6 @@ fn = {"interference": lambda: bench.run_interference(wk, 0, peaks),
       "pressure": lambda: bench.run_pressure(wk, 0),
       "policy": lambda: bench.run_policy_profile(wk, 0),
       "stall_free": lambda: bench.run_stall_free(wk, 0),
-      "handoff": lambda: bench.run_handoff(wk, 0)}[name]
+      "handoff": lambda: bench.run_handoff(wk, 0),
+      "next3": lambda: bench.run_next3(wk, 0, peaks)}[name]
 print(json.dumps(fn()))

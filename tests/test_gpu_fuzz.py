@@ -77,8 +77,8 @@ def test_random_op_matches_oracle(seed):
     lo_min, hi_max = max(fs, fd), min(fs + Ls, fd + Ld)
     lo = int(rng.integers(lo_min, hi_max + 1))
     hi = int(rng.integers(lo, hi_max + 1))
-    mode = rng.choice(["two_pools", "same_pool", "swap_out", "swap_in", "heads"],
-                      p=[0.45, 0.2, 0.1, 0.1, 0.15])
+    mode = rng.choice(["two_pools", "same_pool", "swap_out", "swap_in", "heads", "fanout"],
+                      p=[0.35, 0.2, 0.1, 0.1, 0.15, 0.1])
     kernel = int(rng.choice([wk.KERNEL_TMA, wk.KERNEL_SIMT, wk.KERNEL_COPY_ENGINE], p=[0.45, 0.4, 0.15]))
     big = rng.random() < 0.2                               # a fifth span many CTAs / windows
     nbs, nbd = (int(rng.integers(1, 2000)), int(rng.integers(1, 2000))) if big else \
@@ -118,7 +118,18 @@ def test_random_op_matches_oracle(seed):
     to = (lambda a: torch.as_tensor(a).pin_memory()) if ce else (lambda a: torch.as_tensor(a, device=DEV))
     ts, td = to(sbt), to(dbt)
 
-    if mode == "heads":
+    if mode == "fanout":  # one source table object, k destinations in one launch (NEXT-3)
+        k = int(rng.integers(2, 6))
+        extra = [filled(rng, Ld, H, d, bs, eb, int(rng.integers(n, n + 40)) if n else 1, fd)
+                 for _ in range(k - 1)]
+        tabs = [dbt] + [rng.permutation(p.desc.n_blocks)[:n].astype(np.int32) for p, _ in extra]
+        wk.migrate_batch(src, [(q, ts, to(t), n) for q, t in zip([dst] + [p for p, _ in extra], tabs)], lo, hi)
+        for (q, q0), t in zip(extra, tabs[1:]):
+            w = q0.copy()
+            assert O.migrate(s0, geom(src), sbt, w, geom(q), t, lo, hi) == O.OK
+            assert np.array_equal(read(q), w), dict(fan=k, n=n)
+        assert O.migrate(s0, geom(src), sbt, want, geom(dst), dbt, lo, hi) == O.OK
+    elif mode == "heads":
         sh0 = int(rng.integers(0, H))
         nh = int(rng.integers(1, min(H - sh0, Hd) + 1))
         dh0 = int(rng.integers(0, Hd - nh + 1))

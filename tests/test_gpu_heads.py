@@ -110,3 +110,35 @@ def test_heads_errors_match_oracle():
             got = e.status
         assert got == O.check_op_heads(geom(args[0]), geom(args[1]), 1, 0, 3, s0, d0, nh)
     torch.cuda.synchronize()
+
+
+@pytest.mark.parametrize("k", [2, 3, 4, 5])
+@pytest.mark.parametrize("unit,stages", [(49152, 4), (8192, 6), (65536, 3)])
+@pytest.mark.parametrize("H", [8, 1])
+def test_read_once_fanout(k, unit, stages, H):
+    """NEXT-3 backups, read-once: every batch item passes the SAME source table, so the TMA
+    kernel stages each source unit once and stores it to all k destinations (k <= 4; k = 5
+    takes the per-item path).  Mixed destination tables (one sequential, others shuffled)
+    break runs in some destinations only; whole pools + flags vs the oracle."""
+    wk.set_tuning(wk.PATH_INTRA, kernel=wk.KERNEL_TMA, stage_bytes=unit, stages=stages)
+    rng = np.random.default_rng(100 + k)
+    nb = 90
+    src, s0 = rpool(H, nb, 50)          # C = 32 KiB (parts / 1-2 per unit) or 4 KiB (windows of 16)
+    n = 61
+    sbt = np.sort(rng.permutation(nb)[:n]).astype(np.int32)   # long source runs
+    sbt[::7] = rng.integers(0, nb, sbt[::7].size)              # ... broken, with duplicates
+    ts = tab(sbt)                                              # ONE table object for all items
+    dsts = []
+    for j in range(k):
+        d, d0 = rpool(H, nb + 3 * j, 60 + j)
+        db = (np.arange(n) + j) if j == 0 else rng.permutation(nb + 3 * j)[:n]
+        dsts.append((d, d0, db.astype(np.int32)))
+    n0 = wk.launch_count()
+    wk.migrate_batch(src, [(d, ts, tab(db)) for d, _, db in dsts], 1, 3)
+    torch.cuda.synchronize()
+    assert wk.launch_count() - n0 == 1
+    for d, d0, db in dsts:
+        want = d0.copy()
+        assert O.migrate(s0, geom(src), sbt, want, geom(d), db, 1, 3) == O.OK
+        np.testing.assert_array_equal(d.tensor().cpu().numpy(), want)
+        assert d.layer_ticket() == 1 and [d.layer_count(l) for l in range(3)] == [1, 1, 1]
