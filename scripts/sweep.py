@@ -146,8 +146,32 @@ def compact_sweep():
                               frac=round(2 * gbs / PEAK, 4))), flush=True)
 
 
+def fanout_sweep():
+    """Read-once fan-out (2 and 3 destinations, C2 geometry, half size) over TMA ring shapes."""
+    sh = SHAPES["C2"]
+    case = migration_case("C2", scale=0.5)
+    src = pool(sh, case.nb_src, 1)
+    dsts = [pool(sh, case.nb_dst, 2 + j) for j in range(3)]
+    sbt = torch.as_tensor(case.src_bt, device=dev)
+    dbt = torch.as_tensor(case.dst_bt, device=dev)
+    pb = 2 * sh.n_layers * case.n * sh.chunk_bytes
+    s = torch.cuda.Stream(dev)
+    for k in (2, 3):
+        for stage, stages, lag in [(49152, 4, 2), (49152, 4, 1), (49152, 4, 3), (32768, 6, 3), (32768, 6, 2),
+                                   (32768, 6, 4), (24576, 8, 4), (40960, 5, 2), (65536, 3, 1)]:
+            wk.set_tuning(wk.PATH_INTRA, kernel=wk.KERNEL_TMA, stage_bytes=stage, stages=stages, store_lag=lag,
+                          ctas_per_sm=1)
+            ms = timeit(lambda: wk.migrate_batch(src, [(d, sbt, dbt) for d in dsts[:k]], 0, sh.n_layers,
+                                                 stream=s), s, reps=8)
+            dram = (1 + k) * pb
+            print(json.dumps(dict(case="fanout", k=k, stage_bytes=stage, stages=stages, store_lag=lag,
+                                  ms=round(ms, 3), frac=round(dram / ms / 1e6 / PEAK, 4))), flush=True)
+
+
 def main():
     which = sys.argv[1] if len(sys.argv) > 1 else "all"
+    if which == "fanout":
+        return fanout_sweep()
     if which == "host":
         return host_sweep()
     if which == "compact":
