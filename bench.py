@@ -665,11 +665,14 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     hi_s = torch.cuda.Stream(device, priority=-1)
     lo_s = torch.cuda.Stream(device, priority=0)
 
-    def victim_step():
+    def victim_step_on(st):
         for l in range(sh.n_layers):
             kp = vpool.base + (2 * l) * plane
             victim.decode_attention(q, kp, kp + plane, bt, ctx, sh.n_kv_heads, bs, scratch, out,
-                                    blocks_per_split=bps, stream=hi_s.cuda_stream)
+                                    blocks_per_split=bps, stream=st.cuda_stream)
+
+    def victim_step():
+        victim_step_on(hi_s)
 
     for _ in range(5):
         victim_step()
@@ -681,13 +684,14 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         victim_step()
     torch.cuda.synchronize()
 
-    def victim_run(n):
+    def victim_run(n, g=None, st=None):
+        g, st = g or graph, st or hi_s
         ev = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
-        with torch.cuda.stream(hi_s):
-            ev[0].record(hi_s)
+        with torch.cuda.stream(st):
+            ev[0].record(st)
             for i in range(n):
-                graph.replay()
-                ev[i + 1].record(hi_s)
+                g.replay()
+                ev[i + 1].record(st)
         return ev
     ev = victim_run(n_victim_steps)
     torch.cuda.synchronize()
@@ -711,15 +715,41 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         [(f"rate{r}GBs", {**saved, "max_ctas": 0, "rate_mbps": r * 1000}) for r in (50, 100, 150, 300)] +
         [(f"rate{r}GBs_32ctas", {**saved, "max_ctas": 32, "rate_mbps": r * 1000}) for r in (100,)] +
         [(f"copy_engines_rate{r}GBs", {**saved, "kernel": wk.KERNEL_COPY_ENGINE, "rate_mbps": r * 1000})
-         for r in (50, 100, 150, 300)])
+         for r in (50, 100, 150, 300)] +
+        # SM partition (green contexts, wind_kv_partition_sms): migration confined to 8 SMs,
+        # the victim on the other 140 — no migration CTA ever shares an SM with the victim
+        [("partition8_tma", {**saved, "partition": 8, "max_ctas": 0}),
+         ("partition8_tma_rate50GBs", {**saved, "partition": 8, "max_ctas": 0, "rate_mbps": 50000}),
+         ("partition8_tma_rate150GBs", {**saved, "partition": 8, "max_ctas": 0, "rate_mbps": 150000})])
     rounds, n_round = 3, max(10, n_victim_steps // 2)
+    part = {}  # SM partition (green contexts): victim graph on the compute SMs
+
+    def partitioned(min_sms):
+        if min_sms not in part:
+            P = wk.Partition(device, min_sms)
+            g = torch.cuda.CUDAGraph()
+            for _ in range(2):
+                with torch.cuda.stream(P.compute):
+                    victim_step_on(P.compute)
+            torch.cuda.synchronize()
+            with torch.cuda.graph(g, stream=P.compute):
+                victim_step_on(P.compute)
+            torch.cuda.synchronize()
+            part[min_sms] = (P, g)
+        return part[min_sms]
     for name, cfg in configs:
         cfg = dict(cfg)
         null = cfg.pop("null_feeder", False)  # control: the feeder thread runs, moves nothing
+        min_sms = cfg.pop("partition", 0)
+        mig_s, vic_g, vic_s = lo_s, graph, hi_s
+        if min_sms:
+            P, vic_g = partitioned(min_sms)
+            mig_s, vic_s = P.migration, P.compute
         wk.set_tuning(wk.PATH_INTRA, **cfg)
         ce = cfg.get("kernel") == wk.KERNEL_COPY_ENGINE
         sbt, dbt = (h_tabs[0].data_ptr(), h_tabs[1].data_ptr()) if ce else d_tabs
-        t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, n=case.n, stream=lo_s), 2, 3, lo_s) / 2
+        t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, n=case.n, stream=mig_s), 2, 3, mig_s) / 2
+        full_alone = []
         alone_all, with_all, covered = [], [], True
         # `rounds` interleaved pairs (victim alone, then victim + migration): the alone
         # reference is always adjacent in time (removes clock / power drift).  A feeder
@@ -728,7 +758,11 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         # the host; ctypes releases the GIL inside the library calls).
         for _ in range(rounds):
             torch.cuda.synchronize()
-            ev = victim_run(n_round)
+            if min_sms:  # the whole-GPU reference too: the partition itself costs the victim SMs
+                ev = victim_run(n_round)
+                torch.cuda.synchronize()
+                full_alone += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
+            ev = victim_run(n_round, vic_g, vic_s)
             torch.cuda.synchronize()
             alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
             stop, started, n_ops = threading.Event(), threading.Event(), [0]
@@ -739,14 +773,14 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
                         started.set()
                         time.sleep(0.001)
                         continue
-                    wk.migrate(src, sbt, dst, dbt, n=case.n, stream=lo_s)
+                    wk.migrate(src, sbt, dst, dbt, n=case.n, stream=mig_s)
                     started.set()
-                    lo_s.synchronize()
+                    mig_s.synchronize()
                     n_ops[0] += 1
             th = threading.Thread(target=feeder, daemon=True)
             th.start()
             started.wait()
-            ev = victim_run(n_round)
+            ev = victim_run(n_round, vic_g, vic_s)
             torch.cuda.synchronize()
             stop.set()
             th.join()
@@ -761,7 +795,15 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             "victim_ms_with_migration": round(t_with, 3),
             "slowdown": round(t_with / t_ref - 1.0, 4),
             "migration_covered_all_victim_steps": bool(covered)}
+        if min_sms:
+            t_full = float(np.median(full_alone))
+            res[name].update({"partition_sms_migration": P.sms_migration, "partition_sms_compute": P.sms_compute,
+                              "victim_ms_alone_whole_gpu": round(t_full, 3),
+                              "slowdown_vs_whole_gpu": round(t_with / t_full - 1.0, 4)})
     wk.set_tuning(wk.PATH_INTRA, **saved)
+    torch.cuda.synchronize()
+    for P, _ in part.values():
+        P.destroy()
     del vpool, src, dst
     return res
 

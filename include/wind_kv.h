@@ -294,6 +294,27 @@ wind_status wind_kv_migrate_ex(const wind_kv_pool* src, const int32_t* src_bt, w
                                int32_t layer_hi, const wind_kv_tuning* tuning, void* stream);
 wind_status wind_kv_get_tuning(int32_t path, wind_kv_tuning* t);
 
+/* SM partition (S§7 step 10, interference): two green contexts on `device` with disjoint
+ * SM sets — one of at least `min_sms_migration` SMs (rounded up to the architecture's
+ * granularity: 8 on sm_90+) for migrations, one with the remaining SMs for the co-running
+ * prefill / decode work — and one stream in each (cudaStream_t; migration stream at low
+ * priority, compute stream at high priority).  An op enqueued on the migration stream caps
+ * its grid at that partition's SMs (x ctas_per_sm), and the compute stream's kernels never
+ * share an SM (register file, shared memory, issue slots) with a migration CTA; they still
+ * share HBM / L2 bandwidth.  Errors: INVALID_ARG (NULL out, bad device, min < 1),
+ * UNSUPPORTED (no green-context support in the driver), CUDA.  The caller destroys the
+ * partition after the work on both streams has completed. */
+typedef struct {
+  void* migration_stream;
+  void* compute_stream;
+  int32_t sms_migration;
+  int32_t sms_compute;
+  void* _internal[2];  /* the two green contexts */
+} wind_kv_sm_partition;
+
+wind_status wind_kv_partition_sms(int32_t device, int32_t min_sms_migration, wind_kv_sm_partition* out);
+wind_status wind_kv_partition_destroy(wind_kv_sm_partition* part);
+
 /* Number of kernels this process has launched through the library (all ops). */
 uint64_t wind_kv_launch_count(void);
 

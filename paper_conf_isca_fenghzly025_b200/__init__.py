@@ -22,7 +22,7 @@ __all__ = [
     "WindKVError", "Pool", "lib", "migrate", "migrate_batch", "migrate_heads", "swap_out", "swap_in", "compact",
     "layer_wait", "validate", "plan_compact", "plan_rebalance", "check_device_error",
     "set_tuning", "get_tuning", "launch_count", "STATUS", "PATH_INTRA", "PATH_PEER", "PATH_HOST",
-    "KERNEL_AUTO", "KERNEL_TMA", "KERNEL_SIMT", "EXPORTED_SYMBOLS",
+    "KERNEL_AUTO", "KERNEL_TMA", "KERNEL_SIMT", "EXPORTED_SYMBOLS", "Partition",
 ]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -51,7 +51,7 @@ EXPORTED_SYMBOLS = [
     "wind_kv_plan_rebalance", "wind_kv_check_device_error", "wind_kv_set_tuning",
     "wind_kv_get_tuning", "wind_kv_migrate_ex", "wind_kv_launch_count", "wind_kv_status_string",
     "wind_kv_last_error",
-    "wind_kv_version",
+    "wind_kv_version", "wind_kv_partition_sms", "wind_kv_partition_destroy",
 ]
 
 
@@ -82,6 +82,12 @@ class Tuning(ct.Structure):
     _fields_ = [("kernel", ct.c_int32), ("ctas_per_sm", ct.c_int32), ("stage_bytes", ct.c_int32),
                 ("stages", ct.c_int32), ("max_ctas", ct.c_int32), ("evict_first", ct.c_int32),
                 ("store_lag", ct.c_int32), ("rate_mbps", ct.c_int32)]
+
+
+class SmPartition(ct.Structure):
+    _fields_ = [("migration_stream", ct.c_void_p), ("compute_stream", ct.c_void_p),
+                ("sms_migration", ct.c_int32), ("sms_compute", ct.c_int32),
+                ("_internal", ct.c_void_p * 2)]
 
 
 _LIB: Optional[ct.CDLL] = None
@@ -120,6 +126,8 @@ def lib() -> ct.CDLL:
         "wind_kv_set_tuning": [I32, ct.POINTER(Tuning)],
         "wind_kv_get_tuning": [I32, ct.POINTER(Tuning)],
         "wind_kv_migrate_ex": [P, P, P, P, I32, I32, I32, ct.POINTER(Tuning), P],
+        "wind_kv_partition_sms": [I32, I32, ct.POINTER(SmPartition)],
+        "wind_kv_partition_destroy": [ct.POINTER(SmPartition)],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -422,6 +430,24 @@ def get_tuning(path: int) -> dict:
     t = Tuning()
     _check(lib().wind_kv_get_tuning(path, ct.byref(t)))
     return {k: getattr(t, k) for k, _ in Tuning._fields_}
+
+
+class Partition:
+    """wind_kv_partition_sms: two green contexts with disjoint SM sets on `device` — a
+    migration partition of >= `min_sms` SMs and a compute partition with the rest — and a
+    torch stream in each (`.migration`, `.compute`).  Call destroy() when both are idle."""
+
+    def __init__(self, device: int, min_sms: int):
+        import torch
+        self._p = SmPartition()
+        _check(lib().wind_kv_partition_sms(device, min_sms, ct.byref(self._p)))
+        self.sms_migration, self.sms_compute = self._p.sms_migration, self._p.sms_compute
+        self.migration = torch.cuda.ExternalStream(self._p.migration_stream, device=f"cuda:{device}")
+        self.compute = torch.cuda.ExternalStream(self._p.compute_stream, device=f"cuda:{device}")
+
+    def destroy(self) -> None:
+        if self._p.migration_stream:
+            _check(lib().wind_kv_partition_destroy(ct.byref(self._p)))
 
 
 def launch_count() -> int:

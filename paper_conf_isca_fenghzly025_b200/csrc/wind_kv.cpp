@@ -9,6 +9,7 @@
 #include <stdint.h>
 #include <stdio.h>
 #include <string.h>
+#include <dlfcn.h>
 #include <unistd.h>
 
 #include <algorithm>
@@ -141,6 +142,10 @@ wind_kv_tuning g_tune[3] = {
 }  // namespace
 
 // ---------------------------------------------------------------------------- pool
+
+// Streams of SM partitions (wind_kv_partition_sms, defined at the end of this file): the
+// SM count an op on that stream may use, 0 for any other stream.
+int32_t partition_sms_of(void* stream);
 
 struct wind_kv_pool {
   wind_kv_pool_desc desc;
@@ -762,7 +767,9 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
     return WIND_OK;
   }
-  int64_t grid = static_cast<int64_t>(ctx->sms) * std::max(1, t.ctas_per_sm);
+  // a stream of an SM partition (wind_kv_partition_sms) only has that partition's SMs
+  const int32_t part_sms = partition_sms_of(stream);
+  int64_t grid = static_cast<int64_t>(part_sms > 0 ? part_sms : ctx->sms) * std::max(1, t.ctas_per_sm);
   if (t.max_ctas > 0) grid = std::min<int64_t>(grid, t.max_ctas);
   // A rate-limited op holds as few SMs as can sustain the rate (one CTA moves ~38 GB/s of
   // payload intra-device): the SMs a migration occupies cost a co-running HBM-bound decode
@@ -1060,5 +1067,133 @@ extern "C" const char* wind_kv_status_string(wind_status s) {
 }
 
 extern "C" const char* wind_kv_last_error(void) { return g_last_error.c_str(); }
+
+// ------------------------------------------------------------------ SM partition
+
+namespace {
+
+typedef CUresult (*PFN_deviceGet)(CUdevice*, int);
+typedef CUresult (*PFN_getDevResource)(CUdevice, CUdevResource*, CUdevResourceType);
+typedef CUresult (*PFN_smSplit)(CUdevResource*, unsigned int*, const CUdevResource*, CUdevResource*,
+                                unsigned int, unsigned int);
+typedef CUresult (*PFN_genDesc)(CUdevResourceDesc*, CUdevResource*, unsigned int);
+typedef CUresult (*PFN_greenCreate)(CUgreenCtx*, CUdevResourceDesc, CUdevice, unsigned int);
+typedef CUresult (*PFN_greenDestroy)(CUgreenCtx);
+typedef CUresult (*PFN_greenStream)(CUstream*, CUgreenCtx, unsigned int, int);
+typedef CUresult (*PFN_streamDestroy)(CUstream);
+
+// Driver entry points through the runtime's query, else straight from libcuda.so.1 (the
+// library never links libcuda, so it still loads on a machine without a driver).
+template <typename F>
+F green_fn(const char* name) {
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPointByVersion(name, &fn, 12080, cudaEnableDefault, &q) == cudaSuccess &&
+      q == cudaDriverEntryPointSuccess && fn)
+    return reinterpret_cast<F>(fn);
+  cudaGetLastError();
+  static void* h = dlopen("libcuda.so.1", RTLD_NOW | RTLD_NOLOAD);
+  if (!h) h = dlopen("libcuda.so.1", RTLD_NOW);
+  if (!h) return nullptr;
+  return reinterpret_cast<F>(dlsym(h, name));
+}
+
+}  // namespace
+
+// Streams created by wind_kv_partition_sms and the SM count of their partition (ops on them
+// cap their grid to it; looked up by stream handle).
+std::mutex g_part_mu;
+std::vector<std::pair<void*, int32_t>> g_part_streams;
+
+int32_t partition_sms_of(void* stream) {
+  if (!stream) return 0;
+  std::lock_guard<std::mutex> lk(g_part_mu);
+  for (auto& e : g_part_streams)
+    if (e.first == stream) return e.second;
+  return 0;
+}
+
+extern "C" wind_status wind_kv_partition_sms(int32_t device, int32_t min_sms_migration,
+                                             wind_kv_sm_partition* out) {
+  if (!out || min_sms_migration < 1) return fail(WIND_ERR_INVALID_ARG, "NULL out or min_sms_migration < 1");
+  memset(out, 0, sizeof *out);
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    cudaGetLastError();
+    return fail(WIND_ERR_INVALID_ARG, "bad device %d", device);
+  }
+  auto dget = green_fn<PFN_deviceGet>("cuDeviceGet");
+  auto gres = green_fn<PFN_getDevResource>("cuDeviceGetDevResource");
+  auto split = green_fn<PFN_smSplit>("cuDevSmResourceSplitByCount");
+  auto gdesc = green_fn<PFN_genDesc>("cuDevResourceGenerateDesc");
+  auto gcreate = green_fn<PFN_greenCreate>("cuGreenCtxCreate");
+  auto gdestroy = green_fn<PFN_greenDestroy>("cuGreenCtxDestroy");
+  auto gstream = green_fn<PFN_greenStream>("cuGreenCtxStreamCreate");
+  const char* missing = !dget ? "cuDeviceGet" : !gres ? "cuDeviceGetDevResource" : !split ? "cuDevSmResourceSplitByCount"
+                       : !gdesc ? "cuDevResourceGenerateDesc" : !gcreate ? "cuGreenCtxCreate"
+                       : !gdestroy ? "cuGreenCtxDestroy" : !gstream ? "cuGreenCtxStreamCreate" : nullptr;
+  if (missing) return fail(WIND_ERR_UNSUPPORTED, "driver entry point %s unavailable", missing);
+  DeviceGuard g(device);
+  cudaFree(nullptr);  // the primary context exists (runtime initialised on this device)
+  CUdevice dev;
+  CUresult r = dget(&dev, device);
+  CUdevResource all, grp, rest;
+  memset(&grp, 0, sizeof grp);
+  memset(&rest, 0, sizeof rest);
+  unsigned int ng = 1;
+  if (r == CUDA_SUCCESS) r = gres(dev, &all, CU_DEV_RESOURCE_TYPE_SM);
+  if (r == CUDA_SUCCESS) r = split(&grp, &ng, &all, &rest, 0, static_cast<unsigned int>(min_sms_migration));
+  if (r != CUDA_SUCCESS || ng != 1 || rest.sm.smCount == 0)
+    return fail(WIND_ERR_INVALID_ARG, "cannot split %d SMs off device %d (CUresult %d)", min_sms_migration,
+                device, static_cast<int>(r));
+  CUdevResourceDesc dm, dc;
+  CUgreenCtx gm = nullptr, gc = nullptr;
+  CUstream sm = nullptr, sc = nullptr;
+  r = gdesc(&dm, &grp, 1);
+  if (r == CUDA_SUCCESS) r = gdesc(&dc, &rest, 1);
+  if (r == CUDA_SUCCESS) r = gcreate(&gm, dm, dev, CU_GREEN_CTX_DEFAULT_STREAM);
+  if (r == CUDA_SUCCESS) r = gcreate(&gc, dc, dev, CU_GREEN_CTX_DEFAULT_STREAM);
+  int lo_pri = 0, hi_pri = 0;
+  cudaDeviceGetStreamPriorityRange(&lo_pri, &hi_pri);
+  if (r == CUDA_SUCCESS) r = gstream(&sm, gm, CU_STREAM_NON_BLOCKING, lo_pri);
+  if (r == CUDA_SUCCESS) r = gstream(&sc, gc, CU_STREAM_NON_BLOCKING, hi_pri);
+  if (r != CUDA_SUCCESS) {
+    if (gm) gdestroy(gm);
+    if (gc) gdestroy(gc);
+    return fail(WIND_ERR_CUDA, "green context / stream creation failed (CUresult %d)", static_cast<int>(r));
+  }
+  out->migration_stream = sm;
+  out->compute_stream = sc;
+  out->sms_migration = static_cast<int32_t>(grp.sm.smCount);
+  out->sms_compute = static_cast<int32_t>(rest.sm.smCount);
+  out->_internal[0] = gm;
+  out->_internal[1] = gc;
+  std::lock_guard<std::mutex> lk(g_part_mu);
+  g_part_streams.emplace_back(sm, out->sms_migration);
+  g_part_streams.emplace_back(sc, out->sms_compute);
+  return WIND_OK;
+}
+
+extern "C" wind_status wind_kv_partition_destroy(wind_kv_sm_partition* part) {
+  if (!part) return fail(WIND_ERR_INVALID_ARG, "NULL partition");
+  auto sdestroy = green_fn<PFN_streamDestroy>("cuStreamDestroy");
+  auto gdestroy = green_fn<PFN_greenDestroy>("cuGreenCtxDestroy");
+  if (!sdestroy || !gdestroy) return fail(WIND_ERR_UNSUPPORTED, "green-context entry points unavailable");
+  {
+    std::lock_guard<std::mutex> lk(g_part_mu);
+    g_part_streams.erase(std::remove_if(g_part_streams.begin(), g_part_streams.end(),
+                                        [&](const std::pair<void*, int32_t>& e) {
+                                          return e.first == part->migration_stream ||
+                                                 e.first == part->compute_stream;
+                                        }),
+                         g_part_streams.end());
+  }
+  if (part->migration_stream) sdestroy(static_cast<CUstream>(part->migration_stream));
+  if (part->compute_stream) sdestroy(static_cast<CUstream>(part->compute_stream));
+  for (void* gctx : part->_internal)
+    if (gctx) gdestroy(static_cast<CUgreenCtx>(gctx));
+  memset(part, 0, sizeof *part);
+  return WIND_OK;
+}
 
 extern "C" const char* wind_kv_version(void) { return "wind_kv 0.1.0 (sm_100a)"; }

@@ -33,5 +33,11 @@ fn = {"interference": lambda: bench.run_interference(wk, 0, peaks),
       "policy": lambda: bench.run_policy_profile(wk, 0),
       "stall_free": lambda: bench.run_stall_free(wk, 0),
       "handoff": lambda: bench.run_handoff(wk, 0),
-      "next3": lambda: bench.run_next3(wk, 0, peaks)}[name]
+      "next3": lambda: bench.run_next3(wk, 0, peaks),
+      "partition": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=30, configs=[
+          (n, {**wk.get_tuning(wk.PATH_INTRA), **c}) for n, c in [
+              ("cap8", dict(max_ctas=8)), ("rate50GBs", dict(rate_mbps=50000)),
+              ("partition8_tma", dict(partition=8)), ("partition8_tma_rate50GBs", dict(partition=8, rate_mbps=50000)),
+              ("partition8_tma_rate150GBs", dict(partition=8, rate_mbps=150000)),
+              ("copy_engines_rate50GBs", dict(kernel=3, rate_mbps=50000))]])}[name]
 print(json.dumps(fn()))
