@@ -18,10 +18,12 @@
 // so all CTAs sweep the layers together and a layer completes early (A5 streaming).
 //
 // Layer completion (A5).  When a CTA leaves layer l (its next unit is in a later layer, or
-// it is done) it makes its stores complete and system-visible, then adds 1 to this op's
+// it is done) it makes its stores of l complete and visible, then adds 1 to this op's
 // arrival counter for l; the CTA that brings the counter to gridDim.x publishes
-// dst.layer_done[l] += 1 with a .release.sys reduction (a peer store over NVLink when dst
-// is remote) and resets the counter for the next op using the slot.
+// dst.layer_done[l] += 1 behind a release fence — GPU scope when the data and the flags
+// stay on this GPU, system scope for a peer (NVLink) or host destination — and resets the
+// counter for the next op using the slot.  The TMA consumer defers the arrival until `lag`
+// newer store groups are in flight, so the store pipeline never drains at a layer boundary.
 //
 // Kernels.
 //   tma_copy_kernel  (K2): 2 warps per CTA.  Warp 0 = producer: decodes units and issues
