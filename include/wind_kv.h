@@ -145,8 +145,14 @@ wind_status wind_kv_pool_import(const wind_kv_ipc_handle* handle, int32_t local_
  *     (INVALID_ARG otherwise).  Cross-device ops push over NVLink peer stores (or pull
  *     when src is the remote one); host pools move over PCIe via mapped memory.
  *   Layer flags (A5): every call with n_blocks > 0 and lo < hi takes one ticket on dst
- *     (see wind_kv_layer_ticket) and, as each layer's bytes become visible system-wide,
- *     adds 1 to dst's layer_done flag of that layer; flags of dst layers outside
+ *     (see wind_kv_layer_ticket) and, as each layer's bytes become visible, adds 1 to
+ *     dst's layer_done flag of that layer with release semantics: at GPU scope when src
+ *     and dst are device pools on the executing GPU (every reader of such a pool — the
+ *     consumer stream's wait, the kernels it releases, another process's kernels on that
+ *     GPU — goes through its L2; a system-scope fence per layer cost ~1.7 us),
+ *     at system scope when dst is a peer or host pool.  An agent on another device that
+ *     polls a LOCAL op's flags must order its reads through CUDA events / streams; flags of
+ *     dst layers outside
  *     [lo, hi) are incremented at the start of the op, so "flag >= ticket" is meaningful
  *     for every layer.  Layers are processed in ascending order.
  *   n_blocks == 0 or layer_lo == layer_hi: WIND_OK, nothing enqueued, no ticket (R19). */
