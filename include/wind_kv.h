@@ -25,6 +25,9 @@
  *   - Ops are asynchronous on the given stream, never allocate and never synchronise the
  *     host; they are CUDA-graph capturable.  Asynchronous CUDA faults surface at
  *     the caller's next synchronisation, as with any CUDA call.
+ *   - Each kernel op uses one of 512 per-device arrival-counter slots (round robin): at
+ *     most 512 ops may EXECUTE concurrently on one device across streams (any number may
+ *     be queued on one stream, where ops run in order).
  *   - `cudaStream_t` parameters are passed as `void*` (0 = the legacy default stream) so
  *     the header needs no CUDA include.
  */

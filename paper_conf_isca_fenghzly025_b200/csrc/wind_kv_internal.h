@@ -13,7 +13,7 @@ namespace wkv {
 // Ring of per-op, per-layer CTA-arrival counters on each executing device (A5).  An op
 // takes slot (seq % kCounterSlots); the last CTA to arrive on a layer resets the counter,
 // so a slot is reusable as soon as the op that used it has finished.
-constexpr int kCounterSlots = 64;
+constexpr int kCounterSlots = 512;  // 2 MiB per device; ops in flight CONCURRENTLY (across streams) <= 512
 constexpr int kMaxSegs = 32;  // segments (runs) per work unit = one warp's table window
 constexpr int kMaxFan = 4;    // destinations of a read-once fan-out (TMA kernel)
 constexpr int kCtaMBps = 30000;  // payload MB/s one copy CTA sustains with headroom (~38 measured)
