@@ -136,3 +136,43 @@ def test_plain_c_abi_user():
     out = subprocess.run([exe], capture_output=True, text=True, timeout=300)
     assert out.returncode == 0, out.stderr
     assert "c_abi_example OK" in out.stdout
+
+
+def test_many_concurrent_ops_across_streams():
+    """200 ops enqueued at once on 200 streams (each into its own destination pool), plus
+    a 40-op layer-streamed sequence on one stream: every op takes its own arrival-counter
+    slot; all data byte-exact vs the oracle, every flag == its ticket."""
+    import oracle as O
+    L, H, d, bs, eb = 4, 2, 64, 16, 2
+    rng = np.random.default_rng(7)
+    src = wk.Pool(L, H, d, bs, eb, 64)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    dsts, jobs = [], []
+    for k in range(200):
+        p = wk.Pool(L, H, d, bs, eb, 32)
+        p.tensor().zero_()
+        sbt = rng.permutation(64)[:20].astype(np.int32)
+        dbt = rng.permutation(32)[:20].astype(np.int32)
+        dsts.append(p)
+        jobs.append((p, torch.cuda.Stream(), torch.as_tensor(sbt, device="cuda"),
+                     torch.as_tensor(dbt, device="cuda"), sbt, dbt))
+    torch.cuda.synchronize()
+    for p, st, ts, td, _, _ in jobs:
+        wk.migrate(src, ts, p, td, stream=st)
+    one = wk.Pool(L, H, d, bs, eb, 32)
+    one.tensor().zero_()
+    torch.cuda.synchronize()
+    st1 = torch.cuda.Stream()
+    ts = torch.as_tensor(np.arange(16, dtype=np.int32), device="cuda")
+    for rep in range(10):
+        for l in range(L):
+            wk.migrate(src, ts, one, ts, layer_lo=l, layer_hi=l + 1, stream=st1)
+    torch.cuda.synchronize()
+    g = lambda nb: O.Geom(0, L, H, d, bs, eb, nb)  # noqa: E731
+    for p, _, _, _, sbt, dbt in jobs:
+        want = np.zeros(p.nbytes, np.uint8)
+        assert O.migrate(s0, g(64), sbt, want, g(32), dbt, 0, L) == O.OK
+        np.testing.assert_array_equal(p.tensor().cpu().numpy(), want)
+        assert [p.layer_count(l) for l in range(L)] == [1] * L
+    assert one.layer_ticket() == 40 and [one.layer_count(l) for l in range(L)] == [40] * L
