@@ -70,7 +70,10 @@ typedef enum { WIND_LOC_DEVICE = 0, WIND_LOC_HOST = 1 /* pinned, mapped, portabl
  * Layers are GLOBAL ids [first_layer, first_layer + n_layers) (PP stages).
  * Requirements: every extent >= 1, n_layers <= WIND_KV_MAX_LAYERS, elem_bytes in {1,2,4}
  * (fp8 / fp16|bf16 / fp32 payloads are raw bytes, never interpreted: reading R13),
- * C % 16 == 0.  `device` is ignored for host pools. */
+ * C % 16 == 0.  For a host pool, `device` names the GPU whose copy engines serve it: pool
+ * creation also allocates there the staging of the staged swap path (2 buffers of
+ * max(32 MiB, 2 * n_layers * C) bytes, a side stream, events; best effort — without a GPU
+ * `device` the pool simply has no staging and swaps use the SM kernels). */
 typedef struct {
   int32_t first_layer, n_layers;
   int32_t n_kv_heads, head_dim, block_size, elem_bytes;
@@ -146,7 +149,8 @@ wind_status wind_kv_pool_import(const wind_kv_ipc_handle* handle, int32_t local_
  *   Executing device: src's device if src is a device pool (its own, or the device an
  *     imported src was mapped into), else dst's.  `stream` must belong to it
  *     (INVALID_ARG otherwise).  Cross-device ops push over NVLink peer stores (or pull
- *     when src is the remote one); host pools move over PCIe via mapped memory.
+ *     when src is the remote one); host pools move over PCIe (staged copy engines or
+ *     mapped memory: see wind_kv_swap_out).
  *   Layer flags (A5): every call with n_blocks > 0 and lo < hi takes one ticket on dst
  *     (see wind_kv_layer_ticket) and, as each layer's bytes become visible, adds 1 to
  *     dst's layer_done flag of that layer with release semantics: at GPU scope when src
@@ -165,10 +169,21 @@ wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind
 
 /* swap_out / swap_in (A6): migrate over all layers of the device pool with a HOST pool as
  * destination / source.  The host pool must cover the device pool's
- * layers.  Executes on the device pool's GPU; SM / TMA stores to and loads from mapped
- * pinned memory over PCIe.  A host pool's layer flags live in mapped host memory and are
- * updated without PCIe atomics, so ops INTO one host pool must not overlap in time (ops on
- * one stream never do); the host observes swap_out progress by reading the flags. */
+ * layers.  Executes on the device pool's GPU.  Two mechanisms (HOST path, kernel auto):
+ *   - staged (kernel 4), chosen when the HOST-side table (host_bt) is host-readable (e.g.
+ *     pinned host memory) and the host pool has staging on the executing GPU: a TMA kernel
+ *     gathers (scatters) the device blocks through the device table into a contiguous
+ *     device staging buffer at HBM rate, and the copy engines move each chunk over PCIe,
+ *     one cudaMemcpy2DAsync per run of adjacent host slots, double-buffered on a side
+ *     stream (fork / join with events: graph-capturable).  host_bt is READ ON THE CPU at
+ *     enqueue (entries out of range: BLOCK_RANGE, nothing enqueued).  Staged ops on one
+ *     host pool serialise on its buffers automatically outside graph capture (inside a
+ *     capture, order them yourself).  Layer flags are published once, after all layers.
+ *   - otherwise SM / TMA stores to and loads from mapped pinned memory over PCIe, per-layer
+ *     flags as in migrate.
+ * A host pool's layer flags live in mapped host memory and are updated without PCIe
+ * atomics, so ops INTO one host pool must not overlap in time (ops on one stream never
+ * do); the host observes swap_out progress by reading the flags. */
 wind_status wind_kv_swap_out(const wind_kv_pool* dev, const int32_t* dev_bt,
                              wind_kv_pool* host, const int32_t* host_bt, int32_t n_blocks,
                              void* stream);
@@ -275,9 +290,11 @@ wind_status wind_kv_check_device_error(const wind_kv_pool* pool);
  * of another stream that CUDA maps onto the same queue waits behind them: raise
  * CUDA_DEVICE_MAX_CONNECTIONS (e.g. 32) and keep few streams; the TMA / SIMT kernels pace
  * inside the kernel and never hold a queue),
- * 0 = auto, 1 = TMA bulk staged copy, 2 = SIMT 16-B
- * vector copy.  ctas_per_sm, stage_bytes (TMA stage / SIMT unit bytes, multiple of 16),
- * stages (TMA ring depth); 0 keeps the current value. */
+ * 4 = staged copy engines (HOST path only: see wind_kv_swap_out; UNSUPPORTED when it does
+ * not apply), 0 = auto (INTRA: TMA; PEER: SIMT; HOST: staged when it applies and
+ * rate_mbps == 0, else TMA), 1 = TMA bulk staged copy, 2 = SIMT 16-B vector copy.
+ * ctas_per_sm, stage_bytes (TMA stage / SIMT unit bytes, multiple of 16), stages (TMA ring
+ * depth); 0 keeps the current value. */
 typedef enum { WIND_PATH_INTRA = 0, WIND_PATH_PEER = 1, WIND_PATH_HOST = 2 } wind_path;
 typedef struct {
   int32_t kernel;

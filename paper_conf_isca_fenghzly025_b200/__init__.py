@@ -37,7 +37,7 @@ OK = 0
 LOC_DEVICE, LOC_HOST = 0, 1
 POOL_DEBUG = 0x1
 PATH_INTRA, PATH_PEER, PATH_HOST = 0, 1, 2
-KERNEL_AUTO, KERNEL_TMA, KERNEL_SIMT, KERNEL_COPY_ENGINE = 0, 1, 2, 3
+KERNEL_AUTO, KERNEL_TMA, KERNEL_SIMT, KERNEL_COPY_ENGINE, KERNEL_STAGED = 0, 1, 2, 3, 4
 IPC_HANDLE_BYTES = 512
 MAX_BATCH = 16
 

@@ -136,7 +136,8 @@ wind_kv_tuning g_tune[3] = {
     /* PEER  */ {kSimt, 1, 32768, 6, 96, 0, 0},
     // HOST: PCIe-bound; 8 CTAs reach the same 52 / 51 GB/s as 64 or 148 (sweep r01: SM
     // stores to pinned memory plateau at 0.91 of the copy engines' 57 / 55.5 GB/s)
-    /* HOST  */ {kTma, 1, 49152, 4, 8, 0, 2},
+    // (auto: the staged copy-engine path when the host table is host-readable, staged_host_op)
+    /* HOST  */ {kAuto, 1, 49152, 4, 8, 0, 2},
 };
 
 }  // namespace
@@ -158,6 +159,22 @@ struct wind_kv_pool {
   void* ipc_flags_base = nullptr;
   uint8_t uuid[16] = {};           // physical GPU of the memory (device pools)
   std::atomic<uint32_t> enqueued{0};
+  // Host pools: the staged copy-engine path (kernel 4, staged_host_op).  Two device buffers
+  // on desc.device that SMs gather into / scatter from at HBM rate while the DMA engines
+  // move the other buffer over PCIe, the side stream the DMA runs on, and the events of the
+  // two-buffer pipeline.  Allocated at pool creation; dev < 0 if that failed.
+  struct Staging {
+    int dev = -1;
+    uint8_t* buf[2] = {nullptr, nullptr};
+    size_t buf_bytes = 0;
+    int32_t* iota = nullptr;          // 0, 1, ..., iota_n - 1: the staging side's block table
+    int32_t iota_n = 0;
+    uint32_t* dummy_flags = nullptr;  // layer flags of the internal gather / scatter ops
+    cudaStream_t side = nullptr;
+    cudaEvent_t fork = nullptr, done = nullptr, ready[2] = {nullptr, nullptr},
+                freed[2] = {nullptr, nullptr};
+    bool has_done = false;            // `done` marks the end of the last uncaptured staged op
+  } stg;
 };
 
 namespace {
@@ -181,6 +198,59 @@ wind_status check_desc(const wind_kv_pool_desc* d) {
     return fail(WIND_ERR_UNSUPPORTED, "chunk bytes H*bs*d*e_b = %lld not a multiple of 16",
                 static_cast<long long>(chunk_bytes_of(*d)));
   return WIND_OK;
+}
+
+constexpr size_t kStagingMin = size_t(32) << 20;  // per buffer: >= 0.5 ms of PCIe Gen5 per chunk
+constexpr int32_t kStagingMaxBlocks = 1 << 16;
+
+void staging_free(wind_kv_pool::Staging& g) {
+  if (g.dev < 0) return;
+  DeviceGuard dg(g.dev);
+  for (int b = 0; b < 2; ++b) {
+    if (g.buf[b]) cudaFree(g.buf[b]);
+    if (g.ready[b]) cudaEventDestroy(g.ready[b]);
+    if (g.freed[b]) cudaEventDestroy(g.freed[b]);
+  }
+  if (g.iota) cudaFree(g.iota);
+  if (g.dummy_flags) cudaFree(g.dummy_flags);
+  if (g.fork) cudaEventDestroy(g.fork);
+  if (g.done) cudaEventDestroy(g.done);
+  if (g.side) cudaStreamDestroy(g.side);
+  cudaGetLastError();
+  g = wind_kv_pool::Staging();
+}
+
+// Staging of a host pool on device `dev`: 2 buffers of max(32 MiB, 2 * L * C) bytes (so one
+// block of every layer always fits), the identity table, dummy flags, a side stream and
+// the pipeline events.  Best effort: on failure the pool has no staging and the HOST path
+// uses the SM kernels (mapped pinned memory).
+void staging_init(wind_kv_pool* p, int dev) {
+  wind_kv_pool::Staging& g = p->stg;
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || dev < 0 || dev >= n) {
+    cudaGetLastError();
+    return;
+  }
+  DeviceGuard dg(dev);
+  g.dev = dev;
+  g.buf_bytes = std::max(kStagingMin, static_cast<size_t>(2) * p->desc.n_layers * p->chunk);
+  g.iota_n = static_cast<int32_t>(std::min<int64_t>(kStagingMaxBlocks, g.buf_bytes / (2 * p->chunk)));
+  std::vector<int32_t> iota(g.iota_n);
+  for (int32_t i = 0; i < g.iota_n; ++i) iota[i] = i;
+  bool ok = cudaMalloc(&g.buf[0], g.buf_bytes) == cudaSuccess &&
+            cudaMalloc(&g.buf[1], g.buf_bytes) == cudaSuccess &&
+            cudaMalloc(&g.iota, sizeof(int32_t) * g.iota_n) == cudaSuccess &&
+            cudaMemcpy(g.iota, iota.data(), sizeof(int32_t) * g.iota_n, cudaMemcpyHostToDevice) == cudaSuccess &&
+            cudaMalloc(&g.dummy_flags, sizeof(uint32_t) * WIND_KV_MAX_LAYERS) == cudaSuccess &&
+            cudaMemset(g.dummy_flags, 0, sizeof(uint32_t) * WIND_KV_MAX_LAYERS) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&g.side, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaEventCreateWithFlags(&g.fork, cudaEventDisableTiming) == cudaSuccess &&
+            cudaEventCreateWithFlags(&g.done, cudaEventDisableTiming) == cudaSuccess;
+  for (int b = 0; ok && b < 2; ++b)
+    ok = cudaEventCreateWithFlags(&g.ready[b], cudaEventDisableTiming) == cudaSuccess &&
+         cudaEventCreateWithFlags(&g.freed[b], cudaEventDisableTiming) == cudaSuccess;
+  if (!ok) staging_free(g);
+  cudaGetLastError();
 }
 
 }  // namespace
@@ -261,6 +331,7 @@ extern "C" wind_status wind_kv_pool_create(const wind_kv_pool_desc* desc, void* 
     return fail(WIND_ERR_OOM, "layer flag allocation failed: %s", cudaGetErrorString(e));
   }
   p->owns_flags = true;
+  if (desc->loc == WIND_LOC_HOST) staging_init(p, desc->device);
   *out = p;
   return WIND_OK;
 }
@@ -276,6 +347,7 @@ extern "C" wind_status wind_kv_pool_destroy(wind_kv_pool* p) {
     if (p->owns_data && p->base) cudaFree(p->base);
     if (p->owns_flags && p->flags) cudaFree(p->flags);
   } else {
+    staging_free(p->stg);
     if (p->owns_data && p->base) cudaFreeHost(p->base);
     if (p->owns_flags && p->flags) cudaFreeHost(p->flags);
   }
@@ -621,10 +693,144 @@ wind_status copy_engine_op(const Params& p, const OpItem* items, int n_items, cu
   return WIND_OK;
 }
 
+wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
+                   int32_t hi, void* stream, const HeadRange& hr, const wind_kv_tuning* override_tuning);
+
+// Staged copy-engine host path (kernel 4; the HOST path's automatic choice when the
+// host-side block table is host-readable).  PCIe is the bottleneck of a swap, and the DMA
+// engines drive it harder than SM stores to mapped memory (full-size write packets: 57 vs
+// 52 GB/s D2H on B200, profiles/r01/host_sweep.txt) while holding no SM; but a DMA engine
+// needs every address at enqueue time and pays a setup per copy, so it cannot follow a
+// shuffled device block table.  The op is therefore split by where each side's
+// fragmentation lives:
+//   device side (any table, device-resident): a TMA gather (swap out) / scatter (swap in)
+//     kernel between the device pool and a contiguous staging buffer at HBM rate, 32 CTAs;
+//   host side (table read on the CPU at enqueue): one cudaMemcpy2DAsync per run of adjacent
+//     host slots, rows = the 2 (hi - lo) planes, on a side stream.
+// Chunks of m blocks (m * 2 (hi - lo) * C <= the buffer) alternate between two buffers, so
+// the gather of chunk k + 1 overlaps the PCIe copy of chunk k (fork / join with events:
+// graph-capturable).  The layer flags of dst are published once after the last chunk
+// (like the copy-engine path: no per-layer streaming on this path).
+wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo, int32_t hi,
+                           cudaStream_t s) {
+  const bool out = src->desc.loc == WIND_LOC_DEVICE;  // swap out: device -> host
+  const wind_kv_pool* dev = out ? src : it.dst;
+  const wind_kv_pool* host = out ? it.dst : src;
+  wind_kv_pool::Staging& g = const_cast<wind_kv_pool*>(host)->stg;
+  const int32_t* hbt = out ? it.dbt : it.sbt;       // read here, on the CPU
+  const int32_t* dev_bt = out ? it.sbt : it.dbt;    // read by the gather / scatter kernel
+  const int64_t C = dev->chunk;
+  const int64_t planes = 2LL * (hi - lo);
+  const int32_t m = static_cast<int32_t>(
+      std::min<int64_t>(g.iota_n, static_cast<int64_t>(g.buf_bytes) / (planes * C)));
+  if (m < 1) return fail(WIND_ERR_UNSUPPORTED, "staging buffer smaller than one block of every layer");
+  for (int32_t i = 0; i < it.n; ++i)  // host-side range (the device side is the kernel's contract)
+    if (hbt[i] < 0 || hbt[i] >= host->desc.n_blocks)
+      return fail(WIND_ERR_BLOCK_RANGE, "host block table entry %d = %d out of [0, %d)", i, hbt[i],
+                  host->desc.n_blocks);
+  // the staging buffer seen as a device pool of m blocks over layers [lo, hi), and a shadow
+  // of the device pool: both publish into dummy flags (dst's real flags move once, below)
+  wind_kv_pool stage;
+  stage.desc = dev->desc;
+  stage.desc.first_layer = lo;
+  stage.desc.n_layers = hi - lo;
+  stage.desc.n_blocks = m;
+  stage.desc.flags = 0;
+  stage.chunk = C;
+  stage.bytes = static_cast<size_t>(planes * m * C);
+  stage.flags = g.dummy_flags;
+  memcpy(stage.uuid, dev->uuid, 16);
+  wind_kv_pool shadow;
+  shadow.desc = dev->desc;
+  shadow.desc.flags = 0;
+  shadow.base = dev->base;
+  shadow.chunk = C;
+  shadow.bytes = dev->bytes;
+  shadow.flags = g.dummy_flags;
+  memcpy(shadow.uuid, dev->uuid, 16);
+  // gather / scatter: the intra-device TMA kernel on 32 CTAs (~1.2 TB/s, 20x PCIe)
+  const wind_kv_tuning tg = {kTma, 1, 49152, 4, 32, 0, 2, 0};
+  const int64_t hpitch = static_cast<int64_t>(host->desc.n_blocks) * C;
+  uint8_t* hplane0 = host->base + static_cast<int64_t>(lo - host->desc.first_layer) * 2 * hpitch;
+  const int64_t spitch = static_cast<int64_t>(m) * C;
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(s, &cap) != cudaSuccess) {
+    cudaGetLastError();
+    cap = cudaStreamCaptureStatusNone;
+  }
+  const bool capturing = cap != cudaStreamCaptureStatusNone;
+  // staged ops on one host pool share its buffers: order after the previous one (outside
+  // a graph capture; inside one, the graph's own order applies)
+  if (!capturing && g.has_done) WKV_CUDA(cudaStreamWaitEvent(s, g.done, 0), "cudaStreamWaitEvent(done)");
+  WKV_CUDA(cudaEventRecord(g.fork, s), "cudaEventRecord(fork)");
+  WKV_CUDA(cudaStreamWaitEvent(g.side, g.fork, 0), "cudaStreamWaitEvent(fork)");
+  auto dma = [&](int32_t i0, int32_t mk, uint8_t* buf) -> wind_status {
+    for (int32_t j = i0; j < i0 + mk;) {  // runs of adjacent host slots
+      int32_t r = 1;
+      while (j + r < i0 + mk && hbt[j + r] == hbt[j] + r) ++r;
+      uint8_t* hp = hplane0 + static_cast<int64_t>(hbt[j]) * C;
+      uint8_t* sp = buf + static_cast<int64_t>(j - i0) * C;
+      WKV_CUDA(out ? cudaMemcpy2DAsync(hp, hpitch, sp, spitch, static_cast<size_t>(r * C), planes,
+                                       cudaMemcpyDeviceToHost, g.side)
+                   : cudaMemcpy2DAsync(sp, spitch, hp, hpitch, static_cast<size_t>(r * C), planes,
+                                       cudaMemcpyHostToDevice, g.side),
+               "cudaMemcpy2DAsync(staged)");
+      j += r;
+    }
+    return WIND_OK;
+  };
+  const int32_t K = (it.n + m - 1) / m;
+  wind_status st;
+  for (int32_t k = 0; k < K; ++k) {
+    const int32_t i0 = k * m, mk = std::min(m, it.n - i0), b = k & 1;
+    stage.base = g.buf[b];
+    if (out) {
+      if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(s, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
+      OpItem gi{&stage, dev_bt + i0, g.iota, mk};
+      if ((st = run_op(dev, &gi, 1, lo, hi, s, HeadRange(), &tg)) != WIND_OK) return st;
+      WKV_CUDA(cudaEventRecord(g.ready[b], s), "cudaEventRecord(ready)");
+      WKV_CUDA(cudaStreamWaitEvent(g.side, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
+      if ((st = dma(i0, mk, g.buf[b])) != WIND_OK) return st;
+      WKV_CUDA(cudaEventRecord(g.freed[b], g.side), "cudaEventRecord(freed)");
+    } else {
+      if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(g.side, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
+      if ((st = dma(i0, mk, g.buf[b])) != WIND_OK) return st;
+      WKV_CUDA(cudaEventRecord(g.ready[b], g.side), "cudaEventRecord(ready)");
+      WKV_CUDA(cudaStreamWaitEvent(s, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
+      OpItem si{&shadow, g.iota, dev_bt + i0, mk};
+      if ((st = run_op(&stage, &si, 1, lo, hi, s, HeadRange(), &tg)) != WIND_OK) return st;
+      WKV_CUDA(cudaEventRecord(g.freed[b], s), "cudaEventRecord(freed)");
+    }
+  }
+  if (out)  // join: the side stream's last copy (it runs its work in order)
+    WKV_CUDA(cudaStreamWaitEvent(s, g.freed[(K - 1) & 1], 0), "cudaStreamWaitEvent(join)");
+  // dst's layer flags: every layer once, after all chunks (system scope: a host pool's flags
+  // are read by the CPU; a device pool's by any stream)
+  Params fp;
+  memset(&fp, 0, sizeof fp);
+  fp.n_items = 1;
+  fp.items[0].flags = it.dst->flags;
+  fp.items[0].d_layers = it.dst->desc.n_layers;
+  fp.items[0].host_flags = it.dst->desc.loc == WIND_LOC_HOST;
+  fp.items[0].sys_scope = 1;
+  fp.sys_scope = 1;
+  WKV_CUDA(launch_flag_bump(fp, s), "flag kernel launch");
+  g_launches += 1;
+  if (!capturing) {
+    WKV_CUDA(cudaEventRecord(g.done, s), "cudaEventRecord(done)");
+    g.has_done = true;
+  }
+  it.dst->enqueued.fetch_add(1);
+  return WIND_OK;
+}
+
 // The common op: src -> items[] over layers [lo, hi) on `stream`.
 wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
                    int32_t hi, void* stream, const HeadRange& hr = HeadRange(),
-                   const wind_kv_tuning* override_tuning = nullptr) {
+                   const wind_kv_tuning* override_tuning = nullptr);
+wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
+                   int32_t hi, void* stream, const HeadRange& hr,
+                   const wind_kv_tuning* override_tuning) {
   if (!src) return fail(WIND_ERR_INVALID_ARG, "src pool is NULL");
   if (n_items < 1 || n_items > WIND_KV_MAX_BATCH) return fail(WIND_ERR_INVALID_ARG, "n_items out of range");
   struct NvtxRange {  // one NVTX range per op (the enqueue, on the host timeline)
@@ -670,7 +876,20 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
       debug = true;
     }
 
-  const int kernel = t.kernel == kAuto ? (path == WIND_PATH_INTRA ? kTma : kSimt) : t.kernel;
+  // HOST path, auto: the staged copy-engine path when it applies (one item, whole chunks,
+  // no rate limit, no debug pool, the host pool has staging on this device and its table is
+  // host-readable), else the TMA kernel over mapped pinned memory.
+  if (path == WIND_PATH_HOST && (t.kernel == kStaged || (t.kernel == kAuto && t.rate_mbps == 0))) {
+    const wind_kv_pool* host = src->desc.loc == WIND_LOC_HOST ? src : items[0].dst;
+    const int32_t* hbt = host == src ? items[0].sbt : items[0].dbt;
+    const bool staged = n_items == 1 && hr.n < 0 && !debug && host->stg.dev == exec &&
+                        t.rate_mbps == 0 && host_readable(hbt);
+    if (staged) return staged_host_op(src, items[0], lo, hi, s);
+    if (t.kernel == kStaged)
+      return fail(WIND_ERR_UNSUPPORTED, "staged path needs one item, whole chunks, no rate limit, a "
+                  "host-readable host table and host-pool staging on device %d", exec);
+  }
+  const int kernel = t.kernel == kAuto ? (path == WIND_PATH_PEER ? kSimt : kTma) : t.kernel;
   // Read-once fan-out (backups; NEXT-3): when every item of a batch walks the SAME
   // source table (same pointer and length), the TMA kernel stages each source unit once and
   // stores it to every destination — (1 + k) x payload of DRAM traffic instead of 2k x.
@@ -1001,7 +1220,7 @@ extern "C" wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t)
   if (path < 0 || path > 2 || !t) return fail(WIND_ERR_INVALID_ARG, "bad path or NULL tuning");
   std::lock_guard<std::mutex> lk(g_tune_mu);
   wind_kv_tuning n = g_tune[path];
-  if (t->kernel < 0 || t->kernel > 3) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0, 1, 2 or 3");
+  if (t->kernel < 0 || t->kernel > 4) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0 .. 4");
   n.kernel = t->kernel;
   if (t->ctas_per_sm) n.ctas_per_sm = t->ctas_per_sm;
   if (t->stage_bytes) n.stage_bytes = t->stage_bytes;
@@ -1027,7 +1246,7 @@ extern "C" wind_status wind_kv_migrate_ex(const wind_kv_pool* src, const int32_t
                                           void* stream) {
   if (!dst) return fail(WIND_ERR_INVALID_ARG, "dst pool is NULL");
   if (tuning) {  // validate the override like set_tuning would, then apply it to this op only
-    if (tuning->kernel < 0 || tuning->kernel > 3) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0..3");
+    if (tuning->kernel < 0 || tuning->kernel > 4) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0..4");
     if (tuning->ctas_per_sm < 1 || tuning->ctas_per_sm > 32 || tuning->stage_bytes < 16 ||
         tuning->stage_bytes % 16 || tuning->stages < 3 || tuning->stages > 16 || tuning->store_lag < 0 ||
         tuning->store_lag >= tuning->stages || tuning->rate_mbps < 0 || tuning->max_ctas < 0)

@@ -64,7 +64,7 @@ struct Params {
   Item items[WIND_KV_MAX_BATCH];
 };
 
-enum Kernel { kAuto = 0, kTma = 1, kSimt = 2, kCopyEngine = 3 };
+enum Kernel { kAuto = 0, kTma = 1, kSimt = 2, kCopyEngine = 3, kStaged = 4 };
 
 // Copy-engine path: after the DMA copies of an op (stream-ordered), one tiny kernel adds 1
 // to every layer flag of every item (release, system scope).

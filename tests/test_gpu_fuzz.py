@@ -48,7 +48,7 @@ def read(p: wk.Pool) -> np.ndarray:
 
 
 def draw_tuning(rng, kernel):
-    if kernel == wk.KERNEL_COPY_ENGINE:
+    if kernel in (wk.KERNEL_COPY_ENGINE, wk.KERNEL_STAGED):
         return dict(kernel=kernel, stage_bytes=32768, stages=4)
     unit = int(rng.choice([16, 48, 256, 2048, 4096, 12288, 32768, 49152, 131072]))
     if kernel == wk.KERNEL_TMA:
@@ -80,6 +80,8 @@ def test_random_op_matches_oracle(seed):
     mode = rng.choice(["two_pools", "same_pool", "swap_out", "swap_in", "heads", "fanout"],
                       p=[0.35, 0.2, 0.1, 0.1, 0.15, 0.1])
     kernel = int(rng.choice([wk.KERNEL_TMA, wk.KERNEL_SIMT, wk.KERNEL_COPY_ENGINE], p=[0.45, 0.4, 0.15]))
+    if mode in ("swap_out", "swap_in") and rng.random() < 0.4:
+        kernel = wk.KERNEL_STAGED  # staged copy engines: host-side table read on the CPU
     big = rng.random() < 0.2                               # a fifth span many CTAs / windows
     nbs, nbd = (int(rng.integers(1, 2000)), int(rng.integers(1, 2000))) if big else \
         (int(rng.integers(1, 160)), int(rng.integers(1, 160)))
@@ -114,7 +116,7 @@ def test_random_op_matches_oracle(seed):
         dst, d0 = filled(rng, Ld, Hd, d, bs, eb, nbd, fd, loc=dst_loc)
     flags0 = [dst.layer_count(l) for l in range(fd, fd + Ld)]
     want = d0.copy()
-    ce = kernel == wk.KERNEL_COPY_ENGINE
+    ce = kernel in (wk.KERNEL_COPY_ENGINE, wk.KERNEL_STAGED)  # tables read on the CPU
     to = (lambda a: torch.as_tensor(a).pin_memory()) if ce else (lambda a: torch.as_tensor(a, device=DEV))
     ts, td = to(sbt), to(dbt)
 
