@@ -722,6 +722,12 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     h_tabs = (torch.as_tensor(case.src_bt).pin_memory(), torch.as_tensor(case.dst_bt).pin_memory())
     pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
     saved = wk.get_tuning(wk.PATH_INTRA)
+    saved_host = wk.get_tuning(wk.PATH_HOST)
+    n_sw = min(64, case.n)  # host-swap loads: 64 of the case's blocks (2.25 GiB), looped
+    host = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, n_sw, loc="host")
+    sw_dev = torch.as_tensor(case.src_bt[:n_sw], device=dev)
+    sw_host = {"dev": torch.arange(n_sw, dtype=torch.int32, device=dev),
+               "pinned": torch.arange(n_sw, dtype=torch.int32).pin_memory()}
     configs = configs or (
         [("control_no_migration", {**saved, "null_feeder": True})] +
         [(f"cap{c or 'none'}", {**saved, "max_ctas": c}) for c in (2, 4, 8, 16, 0)] +
@@ -733,7 +739,16 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         # the victim on the other 140 — no migration CTA ever shares an SM with the victim
         [("partition8_tma", {**saved, "partition": 8, "max_ctas": 0}),
          ("partition8_tma_rate50GBs", {**saved, "partition": 8, "max_ctas": 0, "rate_mbps": 50000}),
-         ("partition8_tma_rate150GBs", {**saved, "partition": 8, "max_ctas": 0, "rate_mbps": 150000})])
+         ("partition8_tma_rate150GBs", {**saved, "partition": 8, "max_ctas": 0, "rate_mbps": 150000})] +
+        # host swaps (A6) next to the decode victim: the SM kernel on mapped pinned memory (HBM
+        # one way only: swap out reads, swap in writes) at the library's per-direction CTA
+        # defaults, the swap-out at the former 8-CTA default (PCIe write backpressure), and the
+        # staged copy-engine path (gather / scatter through the staging buffer + DMA)
+        [("swap_out_sm_default", {"op": "swap_out", **saved_host, "kernel": wk.KERNEL_TMA}),
+         ("swap_out_sm_8ctas", {"op": "swap_out", **saved_host, "kernel": wk.KERNEL_TMA, "max_ctas": 8}),
+         ("swap_in_sm_default", {"op": "swap_in", **saved_host, "kernel": wk.KERNEL_TMA}),
+         ("swap_out_staged", {"op": "swap_out", **saved_host, "kernel": wk.KERNEL_STAGED}),
+         ("swap_in_staged", {"op": "swap_in", **saved_host, "kernel": wk.KERNEL_STAGED})])
     rounds, n_round = 3, max(10, n_victim_steps // 2)
     part = {}  # SM partition (green contexts): victim graph on the compute SMs
 
@@ -754,14 +769,30 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         cfg = dict(cfg)
         null = cfg.pop("null_feeder", False)  # control: the feeder thread runs, moves nothing
         min_sms = cfg.pop("partition", 0)
+        op_kind = cfg.pop("op", "migrate")
         mig_s, vic_g, vic_s = lo_s, graph, hi_s
         if min_sms:
             P, vic_g = partitioned(min_sms)
             mig_s, vic_s = P.migration, P.compute
-        wk.set_tuning(wk.PATH_INTRA, **cfg)
-        ce = cfg.get("kernel") == wk.KERNEL_COPY_ENGINE
-        sbt, dbt = (h_tabs[0].data_ptr(), h_tabs[1].data_ptr()) if ce else d_tabs
-        t_mig = time_device(lambda: wk.migrate(src, sbt, dst, dbt, n=case.n, stream=mig_s), 2, 3, mig_s) / 2
+        if op_kind == "migrate":
+            wk.set_tuning(wk.PATH_INTRA, **cfg)
+            ce = cfg.get("kernel") == wk.KERNEL_COPY_ENGINE
+            sbt, dbt = (h_tabs[0].data_ptr(), h_tabs[1].data_ptr()) if ce else d_tabs
+            op_bytes = pb
+
+            def one_op():
+                wk.migrate(src, sbt, dst, dbt, n=case.n, stream=mig_s)
+        else:
+            wk.set_tuning(wk.PATH_HOST, **cfg)
+            ht = sw_host["pinned" if cfg.get("kernel") == wk.KERNEL_STAGED else "dev"]
+            op_bytes = payload_bytes(n_sw, sh.n_layers, sh.chunk_bytes)
+            if op_kind == "swap_out":
+                def one_op():
+                    wk.swap_out(src, sw_dev, host, ht, stream=mig_s)
+            else:
+                def one_op():
+                    wk.swap_in(host, ht, src, sw_dev, stream=mig_s)
+        t_mig = time_device(one_op, 2, 3, mig_s) / 2
         full_alone = []
         alone_all, with_all, covered = [], [], True
         # `rounds` interleaved pairs (victim alone, then victim + migration): the alone
@@ -786,7 +817,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
                         started.set()
                         time.sleep(0.001)
                         continue
-                    wk.migrate(src, sbt, dst, dbt, n=case.n, stream=mig_s)
+                    one_op()
                     started.set()
                     mig_s.synchronize()
                     n_ops[0] += 1
@@ -801,9 +832,12 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             with_all += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
             alone_all += alone
         t_ref, t_with = float(np.median(alone_all)), float(np.median(with_all))
+        # HBM bytes per payload byte: intra-device read + write; SM swap one way; the staged
+        # swap adds its gather / scatter through the staging buffer (3 ways)
+        hbm_ways = 2 if op_kind == "migrate" else (3 if cfg.get("kernel") == wk.KERNEL_STAGED else 1)
         res[name] = {
-            "migration_gbs_alone": round(pb / t_mig / 1e6, 1),
-            "migration_hbm_share": round(2 * pb / t_mig / 1e6 / peaks["hbm_gbs"], 4),
+            "migration_gbs_alone": round(op_bytes / t_mig / 1e6, 1),
+            "migration_hbm_share": round(hbm_ways * op_bytes / t_mig / 1e6 / peaks["hbm_gbs"], 4),
             "victim_ms_alone_adjacent": round(t_ref, 3),
             "victim_ms_with_migration": round(t_with, 3),
             "slowdown": round(t_with / t_ref - 1.0, 4),
@@ -814,9 +848,11 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
                               "victim_ms_alone_whole_gpu": round(t_full, 3),
                               "slowdown_vs_whole_gpu": round(t_with / t_full - 1.0, 4)})
     wk.set_tuning(wk.PATH_INTRA, **saved)
+    wk.set_tuning(wk.PATH_HOST, **saved_host)
     torch.cuda.synchronize()
     for P, _ in part.values():
         P.destroy()
+    host.destroy()
     del vpool, src, dst
     return res
 

@@ -301,7 +301,13 @@ typedef struct {
   int32_t ctas_per_sm;
   int32_t stage_bytes;
   int32_t stages;
-  int32_t max_ctas; /* cap on the grid (e.g. to leave SMs to a decode stream); 0 = none */
+  int32_t max_ctas; /* cap on the grid (e.g. to leave SMs to a decode stream); 0 = none,
+                       except on the HOST path where 0 = per-direction defaults: SM kernel
+                       into host memory with ~384 KiB of stores in flight (2-3 CTAs; more
+                       back PCIe writes up into the GPU's memory system: 1.5 MiB in flight
+                       slowed a co-running decode kernel by 73 %, 384 KiB by 2 %, same
+                       52 GB/s), 8 CTAs from host memory; staged path: hidden gather /
+                       scatter chunks with ~768 KiB in flight (4-6 CTAs) */
   int32_t evict_first; /* 1 = L2 evict-first policy on the copy's loads and stores */
   int32_t store_lag;   /* TMA: stores allowed in flight per CTA (0 = stages / 2) */
   int32_t rate_mbps;   /* payload rate limit of one op in MB/s (0 = unlimited): bounds the

@@ -134,11 +134,41 @@ wind_kv_tuning g_tune[3] = {
     // threads keep ~3 MiB of stores in flight (> 2 us x 900 GB/s) and leave SMs to the
     // co-running prefill / decode.  Not yet tuned on a multi-GPU box (one GPU per round-1 call).
     /* PEER  */ {kSimt, 1, 32768, 6, 96, 0, 0},
-    // HOST: PCIe-bound; 8 CTAs reach the same 52 / 51 GB/s as 64 or 148 (sweep r01: SM
-    // stores to pinned memory plateau at 0.91 of the copy engines' 57 / 55.5 GB/s)
-    // (auto: the staged copy-engine path when the host table is host-readable, staged_host_op)
-    /* HOST  */ {kAuto, 1, 49152, 4, 8, 0, 2},
+    // HOST: PCIe-bound.  auto = the staged copy-engine path when the host table is
+    // host-readable (staged_host_op), else the TMA kernel on mapped pinned memory.
+    // max_ctas 0 = per-direction defaults (kHostCtas*): SM stores to host memory beyond
+    // what PCIe drains back up into the GPU's memory system — 8 TMA CTAs writing at 52 GB/s
+    // slowed a co-running decode kernel by 73 %, 2 CTAs at the same rate by 2 %
+    /* HOST  */ {kAuto, 1, 49152, 4, 0, 0, 2},
 };
+
+// HOST path defaults when the tuning's max_ctas is 0 (sweep r01: scripts/staged_sweep.py and
+// the bench's c3_interference swap rows, profiles/r01/interference_swap_sweep*.json).  What
+// matters is the bytes a grid keeps in flight (stages x work-unit bytes per CTA):
+//  - SM stores into host memory: ~384 KiB in flight saturates PCIe (52 GB/s) and costs a
+//    co-running decode kernel 2 %; 576 KiB 5 %, 768 KiB 7 %, 1.5 MiB 73 % (the writes PCIe
+//    cannot drain back up into the GPU's memory system);
+//  - SM loads from host memory: 8 CTAs (51 GB/s; fewer lose rate on small chunks);
+//  - staged gather / scatter chunks hidden behind PCIe copies: ~768 KiB in flight keeps
+//    them ahead of PCIe (56-57 / 55 GB/s) with 4-6 % victim cost (1.5 MiB+: no faster).
+constexpr int64_t kHostToHostInFlight = 384 << 10;
+constexpr int kHostCtasFromHost = 8;
+constexpr int64_t kStagedInFlight = 768 << 10;
+
+// Bytes one work unit covers for copies of CP bytes per block with units of at most `unit`
+// bytes (the decomposition run_op gives the kernels).
+int64_t work_unit_bytes(int64_t CP, int64_t unit) {
+  if (CP >= unit) {
+    const int64_t parts = (CP + unit - 1) / unit;
+    return ((CP + parts - 1) / parts + 15) / 16 * 16;
+  }
+  return std::min<int64_t>(kMaxSegs, unit / CP) * CP;
+}
+
+int ctas_for_in_flight(int64_t target, int stages, int64_t unit_bytes) {
+  const int64_t per_cta = std::max<int64_t>(1, static_cast<int64_t>(stages) * unit_bytes);
+  return static_cast<int>(std::max<int64_t>(1, (target + per_cta - 1) / per_cta));
+}
 
 }  // namespace
 
@@ -712,7 +742,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
 // graph-capturable).  The layer flags of dst are published once after the last chunk
 // (like the copy-engine path: no per-layer streaming on this path).
 wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo, int32_t hi,
-                           cudaStream_t s) {
+                           cudaStream_t s, int32_t hidden_ctas) {
   const bool out = src->desc.loc == WIND_LOC_DEVICE;  // swap out: device -> host
   const wind_kv_pool* dev = out ? src : it.dst;
   const wind_kv_pool* host = out ? it.dst : src;
@@ -748,8 +778,12 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
   shadow.bytes = dev->bytes;
   shadow.flags = g.dummy_flags;
   memcpy(shadow.uuid, dev->uuid, 16);
-  // gather / scatter: the intra-device TMA kernel on 32 CTAs (~1.2 TB/s, 20x PCIe)
-  const wind_kv_tuning tg = {kTma, 1, 49152, 4, 32, 0, 2, 0};
+  // gather / scatter: the intra-device TMA kernel.  The one chunk whose gather (swap out:
+  // the first) or scatter (swap in: the last) is not hidden behind a PCIe copy runs on every
+  // SM (~10 us per 32 MiB); the hidden ones on `hidden_ctas` CTAs (~38 GB/s each: 8 CTAs
+  // stay ~5x ahead of PCIe) so they take few SMs and little HBM burst from co-running work.
+  const wind_kv_tuning t_exposed = {kTma, 1, 49152, 4, 0, 0, 2, 0};
+  const wind_kv_tuning t_hidden = {kTma, 1, 49152, 4, std::max(1, hidden_ctas), 0, 2, 0};
   const int64_t hpitch = static_cast<int64_t>(host->desc.n_blocks) * C;
   uint8_t* hplane0 = host->base + static_cast<int64_t>(lo - host->desc.first_layer) * 2 * hpitch;
   const int64_t spitch = static_cast<int64_t>(m) * C;
@@ -787,7 +821,8 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
     if (out) {
       if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(s, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
       OpItem gi{&stage, dev_bt + i0, g.iota, mk};
-      if ((st = run_op(dev, &gi, 1, lo, hi, s, HeadRange(), &tg)) != WIND_OK) return st;
+      if ((st = run_op(dev, &gi, 1, lo, hi, s, HeadRange(), k == 0 ? &t_exposed : &t_hidden)) != WIND_OK)
+        return st;
       WKV_CUDA(cudaEventRecord(g.ready[b], s), "cudaEventRecord(ready)");
       WKV_CUDA(cudaStreamWaitEvent(g.side, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
       if ((st = dma(i0, mk, g.buf[b])) != WIND_OK) return st;
@@ -798,7 +833,8 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
       WKV_CUDA(cudaEventRecord(g.ready[b], g.side), "cudaEventRecord(ready)");
       WKV_CUDA(cudaStreamWaitEvent(s, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
       OpItem si{&shadow, g.iota, dev_bt + i0, mk};
-      if ((st = run_op(&stage, &si, 1, lo, hi, s, HeadRange(), &tg)) != WIND_OK) return st;
+      if ((st = run_op(&stage, &si, 1, lo, hi, s, HeadRange(), k == K - 1 ? &t_exposed : &t_hidden)) != WIND_OK)
+        return st;
       WKV_CUDA(cudaEventRecord(g.freed[b], s), "cudaEventRecord(freed)");
     }
   }
@@ -884,7 +920,10 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     const int32_t* hbt = host == src ? items[0].sbt : items[0].dbt;
     const bool staged = n_items == 1 && hr.n < 0 && !debug && host->stg.dev == exec &&
                         t.rate_mbps == 0 && host_readable(hbt);
-    if (staged) return staged_host_op(src, items[0], lo, hi, s);
+    if (staged)  // hidden chunks run the staged kernel tuning (4 x 48 KiB stages)
+      return staged_host_op(src, items[0], lo, hi, s,
+                            t.max_ctas > 0 ? t.max_ctas
+                                           : ctas_for_in_flight(kStagedInFlight, 4, work_unit_bytes(src->chunk, 49152)));
     if (t.kernel == kStaged)
       return fail(WIND_ERR_UNSUPPORTED, "staged path needs one item, whole chunks, no rate limit, a "
                   "host-readable host table and host-pool staging on device %d", exec);
@@ -989,7 +1028,15 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   // a stream of an SM partition (wind_kv_partition_sms) only has that partition's SMs
   const int32_t part_sms = partition_sms_of(stream);
   int64_t grid = static_cast<int64_t>(part_sms > 0 ? part_sms : ctx->sms) * std::max(1, t.ctas_per_sm);
-  if (t.max_ctas > 0) grid = std::min<int64_t>(grid, t.max_ctas);
+  if (t.max_ctas > 0)
+    grid = std::min<int64_t>(grid, t.max_ctas);
+  else if (path == WIND_PATH_HOST) {
+    bool to_host = false;  // any store into host memory: the backpressure-prone direction
+    for (int j = 0; j < n_items; ++j) to_host = to_host || items[j].dst->desc.loc == WIND_LOC_HOST;
+    grid = std::min<int64_t>(grid, to_host ? ctas_for_in_flight(kHostToHostInFlight, t.stages,
+                                                                work_unit_bytes(CP, t.stage_bytes))
+                                           : kHostCtasFromHost);
+  }
   // A rate-limited op holds as few SMs as can sustain the rate (one CTA moves ~38 GB/s of
   // payload intra-device): the SMs a migration occupies cost a co-running HBM-bound decode
   // kernel more than the bytes it moves (bench c3_interference).

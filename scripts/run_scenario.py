@@ -30,6 +30,50 @@ fn = {"interference": lambda: bench.run_interference(wk, 0, peaks),
       "interference_configs": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=30,
                                                              configs=small_footprint),
       "pressure": lambda: bench.run_pressure(wk, 0),
+      "interference_rw": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=40, configs=[
+          (n, c) for n, c in [
+              ("control_no_migration", {**wk.get_tuning(wk.PATH_INTRA), "null_feeder": True}),
+              ("rate50GBs", {**wk.get_tuning(wk.PATH_INTRA), "rate_mbps": 50000}),
+              ("rate50GBs_evict_first", {**wk.get_tuning(wk.PATH_INTRA), "rate_mbps": 50000, "evict_first": 1}),
+              ("copy_engines_rate50GBs", {**wk.get_tuning(wk.PATH_INTRA), "kernel": 3, "rate_mbps": 50000}),
+              ("hbm_reads_only_swap_out_sm8", {"op": "swap_out", **wk.get_tuning(wk.PATH_HOST), "kernel": 1}),
+              ("hbm_writes_only_swap_in_sm8", {"op": "swap_in", **wk.get_tuning(wk.PATH_HOST), "kernel": 1}),
+              ("swap_out_staged_ce", {"op": "swap_out", **wk.get_tuning(wk.PATH_HOST), "kernel": 4}),
+              ("swap_in_staged_ce", {"op": "swap_in", **wk.get_tuning(wk.PATH_HOST), "kernel": 4}),
+              ("hbm_reads_only_swap_out_sm8_b", {"op": "swap_out", **wk.get_tuning(wk.PATH_HOST), "kernel": 1}),
+              ("hbm_writes_only_swap_in_sm8_b", {"op": "swap_in", **wk.get_tuning(wk.PATH_HOST), "kernel": 1}),
+          ]]),
+      "interference_swap": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=40, configs=[
+          (n, {"op": op, **wk.get_tuning(wk.PATH_HOST), **c}) for n, op, c in [
+              ("staged_out_default", "swap_out", dict(kernel=4)),
+              ("staged_in_default", "swap_in", dict(kernel=4)),
+              ("staged_out_hidden2", "swap_out", dict(kernel=4, max_ctas=2)),
+              ("staged_out_hidden32", "swap_out", dict(kernel=4, max_ctas=32)),
+              ("sm_out_tma8", "swap_out", dict(kernel=1)),
+              ("sm_out_tma8_rate45", "swap_out", dict(kernel=1, rate_mbps=45000)),
+              ("sm_out_tma8_rate30", "swap_out", dict(kernel=1, rate_mbps=30000)),
+              ("sm_out_tma2", "swap_out", dict(kernel=1, max_ctas=2)),
+              ("sm_out_tma1", "swap_out", dict(kernel=1, max_ctas=1)),
+              ("sm_out_simt8", "swap_out", dict(kernel=2, max_ctas=8, stage_bytes=32768)),
+              ("sm_out_simt2", "swap_out", dict(kernel=2, max_ctas=2, stage_bytes=32768)),
+              ("sm_in_tma8", "swap_in", dict(kernel=1)),
+          ]]),
+      "interference_swap2": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=40, configs=[
+          (n, {"op": op, **wk.get_tuning(wk.PATH_HOST), **c}) for n, op, c in [
+              ("staged_out_h4", "swap_out", dict(kernel=4, max_ctas=4)),
+              ("staged_in_h4", "swap_in", dict(kernel=4, max_ctas=4)),
+              ("staged_out_h2", "swap_out", dict(kernel=4, max_ctas=2)),
+              ("staged_in_h2", "swap_in", dict(kernel=4, max_ctas=2)),
+              ("sm_out_tma2", "swap_out", dict(kernel=1, max_ctas=2)),
+              ("sm_out_tma3", "swap_out", dict(kernel=1, max_ctas=3)),
+              ("sm_out_tma4", "swap_out", dict(kernel=1, max_ctas=4)),
+              ("sm_out_tma8_rate50", "swap_out", dict(kernel=1, max_ctas=8, rate_mbps=50000)),
+              ("sm_in_tma2", "swap_in", dict(kernel=1, max_ctas=2)),
+              ("sm_in_tma4", "swap_in", dict(kernel=1, max_ctas=4)),
+              ("sm_in_tma8", "swap_in", dict(kernel=1, max_ctas=8)),
+              ("staged_out_h4_b", "swap_out", dict(kernel=4, max_ctas=4)),
+              ("sm_out_tma2_b", "swap_out", dict(kernel=1, max_ctas=2)),
+          ]]),
       "policy": lambda: bench.run_policy_profile(wk, 0),
       "stall_free": lambda: bench.run_stall_free(wk, 0),
       "handoff": lambda: bench.run_handoff(wk, 0),
