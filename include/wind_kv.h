@@ -175,10 +175,11 @@ wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind
  *     gathers (scatters) the device blocks through the device table into a contiguous
  *     device staging buffer at HBM rate, and the copy engines move each chunk over PCIe,
  *     one cudaMemcpy2DAsync per run of adjacent host slots, double-buffered on a side
- *     stream (fork / join with events: graph-capturable).  host_bt is READ ON THE CPU at
- *     enqueue (entries out of range: BLOCK_RANGE, nothing enqueued).  Staged ops on one
- *     host pool serialise on its buffers automatically outside graph capture (inside a
- *     capture, order them yourself).  Layer flags are published once, after all layers.
+ *     stream (fork / join with events: graph-capturable).  Chunks are layer-major and
+ *     dst's layer flags move as each layer's last chunk lands (layer_wait works as for
+ *     migrate).  host_bt is READ ON THE CPU at enqueue (entries out of range: BLOCK_RANGE,
+ *     nothing enqueued).  Staged ops on one host pool serialise on its buffers
+ *     automatically outside graph capture (inside a capture, order them yourself).
  *   - otherwise SM / TMA stores to and loads from mapped pinned memory over PCIe, per-layer
  *     flags as in migrate.
  * A host pool's layer flags live in mapped host memory and are updated without PCIe

@@ -734,13 +734,16 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
 // shuffled device block table.  The op is therefore split by where each side's
 // fragmentation lives:
 //   device side (any table, device-resident): a TMA gather (swap out) / scatter (swap in)
-//     kernel between the device pool and a contiguous staging buffer at HBM rate, 32 CTAs;
+//     kernel between the device pool and a contiguous staging buffer at HBM rate;
 //   host side (table read on the CPU at enqueue): one cudaMemcpy2DAsync per run of adjacent
-//     host slots, rows = the 2 (hi - lo) planes, on a side stream.
-// Chunks of m blocks (m * 2 (hi - lo) * C <= the buffer) alternate between two buffers, so
-// the gather of chunk k + 1 overlaps the PCIe copy of chunk k (fork / join with events:
-// graph-capturable).  The layer flags of dst are published once after the last chunk
-// (like the copy-engine path: no per-layer streaming on this path).
+//     host slots, rows = the chunk's K/V planes, on a side stream.
+// Chunks are layer-major (A5): a chunk is a range of whole layers for all n blocks
+// when they fit the buffer, else one layer for a range of blocks.  They alternate between
+// two buffers, so the gather of chunk k + 1 overlaps the PCIe copy of chunk k (fork / join
+// with events: graph-capturable).  dst's layer flags are published as each layer's last
+// chunk lands (after its PCIe copy on the side stream for a swap out, after its scatter on
+// the op's stream for a swap in), so a consumer can start on layer 0 of a swap-in while
+// later layers are still in flight.
 wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo, int32_t hi,
                            cudaStream_t s, int32_t hidden_ctas) {
   const bool out = src->desc.loc == WIND_LOC_DEVICE;  // swap out: device -> host
@@ -750,24 +753,26 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
   const int32_t* hbt = out ? it.dbt : it.sbt;       // read here, on the CPU
   const int32_t* dev_bt = out ? it.sbt : it.dbt;    // read by the gather / scatter kernel
   const int64_t C = dev->chunk;
-  const int64_t planes = 2LL * (hi - lo);
-  const int32_t m = static_cast<int32_t>(
-      std::min<int64_t>(g.iota_n, static_cast<int64_t>(g.buf_bytes) / (planes * C)));
-  if (m < 1) return fail(WIND_ERR_UNSUPPORTED, "staging buffer smaller than one block of every layer");
+  const int64_t layer_bytes = 2 * C * static_cast<int64_t>(it.n);  // one layer, all blocks
+  // chunk shape: whole layers x all blocks when one layer fits, else 1 layer x m blocks
+  int32_t lpc = 1, m = it.n;
+  if (it.n <= g.iota_n && layer_bytes <= static_cast<int64_t>(g.buf_bytes)) {
+    lpc = static_cast<int32_t>(std::min<int64_t>(hi - lo, static_cast<int64_t>(g.buf_bytes) / layer_bytes));
+  } else {
+    m = static_cast<int32_t>(std::min<int64_t>(g.iota_n, static_cast<int64_t>(g.buf_bytes) / (2 * C)));
+    if (m < 1) return fail(WIND_ERR_UNSUPPORTED, "staging buffer smaller than one block of one layer");
+  }
   for (int32_t i = 0; i < it.n; ++i)  // host-side range (the device side is the kernel's contract)
     if (hbt[i] < 0 || hbt[i] >= host->desc.n_blocks)
       return fail(WIND_ERR_BLOCK_RANGE, "host block table entry %d = %d out of [0, %d)", i, hbt[i],
                   host->desc.n_blocks);
-  // the staging buffer seen as a device pool of m blocks over layers [lo, hi), and a shadow
-  // of the device pool: both publish into dummy flags (dst's real flags move once, below)
+  // the staging buffer seen as a device pool of m blocks over a chunk's layers, and a shadow
+  // of the device pool: both publish into dummy flags (dst's real flags: flag_range below)
   wind_kv_pool stage;
   stage.desc = dev->desc;
-  stage.desc.first_layer = lo;
-  stage.desc.n_layers = hi - lo;
   stage.desc.n_blocks = m;
   stage.desc.flags = 0;
   stage.chunk = C;
-  stage.bytes = static_cast<size_t>(planes * m * C);
   stage.flags = g.dummy_flags;
   memcpy(stage.uuid, dev->uuid, 16);
   wind_kv_pool shadow;
@@ -780,13 +785,27 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
   memcpy(shadow.uuid, dev->uuid, 16);
   // gather / scatter: the intra-device TMA kernel.  The one chunk whose gather (swap out:
   // the first) or scatter (swap in: the last) is not hidden behind a PCIe copy runs on every
-  // SM (~10 us per 32 MiB); the hidden ones on `hidden_ctas` CTAs (~38 GB/s each: 8 CTAs
-  // stay ~5x ahead of PCIe) so they take few SMs and little HBM burst from co-running work.
+  // SM (~10 us per 32 MiB); the hidden ones on `hidden_ctas` CTAs so they take few SMs and
+  // little HBM burst from co-running work.
   const wind_kv_tuning t_exposed = {kTma, 1, 49152, 4, 0, 0, 2, 0};
   const wind_kv_tuning t_hidden = {kTma, 1, 49152, 4, std::max(1, hidden_ctas), 0, 2, 0};
   const int64_t hpitch = static_cast<int64_t>(host->desc.n_blocks) * C;
-  uint8_t* hplane0 = host->base + static_cast<int64_t>(lo - host->desc.first_layer) * 2 * hpitch;
   const int64_t spitch = static_cast<int64_t>(m) * C;
+  // +1 on dst's layer_done flags [a, b) (global ids), system scope, on stream `st`
+  auto flag_range = [&](int32_t a, int32_t b, cudaStream_t st) -> wind_status {
+    if (a >= b) return WIND_OK;
+    Params fp;
+    memset(&fp, 0, sizeof fp);
+    fp.n_items = 1;
+    fp.items[0].flags = it.dst->flags + (a - it.dst->desc.first_layer);
+    fp.items[0].d_layers = b - a;
+    fp.items[0].host_flags = it.dst->desc.loc == WIND_LOC_HOST;
+    fp.items[0].sys_scope = 1;
+    fp.sys_scope = 1;
+    WKV_CUDA(launch_flag_bump(fp, st), "flag kernel launch");
+    g_launches += 1;
+    return WIND_OK;
+  };
   cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
   if (cudaStreamIsCapturing(s, &cap) != cudaSuccess) {
     cudaGetLastError();
@@ -796,62 +815,67 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
   // staged ops on one host pool share its buffers: order after the previous one (outside
   // a graph capture; inside one, the graph's own order applies)
   if (!capturing && g.has_done) WKV_CUDA(cudaStreamWaitEvent(s, g.done, 0), "cudaStreamWaitEvent(done)");
+  wind_status st;
+  // dst layers outside [lo, hi): +1 at the start, as every op does (wind_kv_migrate)
+  const int32_t f0 = it.dst->desc.first_layer, f1 = f0 + it.dst->desc.n_layers;
+  if ((st = flag_range(f0, lo, s)) != WIND_OK) return st;
+  if ((st = flag_range(hi, f1, s)) != WIND_OK) return st;
   WKV_CUDA(cudaEventRecord(g.fork, s), "cudaEventRecord(fork)");
   WKV_CUDA(cudaStreamWaitEvent(g.side, g.fork, 0), "cudaStreamWaitEvent(fork)");
-  auto dma = [&](int32_t i0, int32_t mk, uint8_t* buf) -> wind_status {
-    for (int32_t j = i0; j < i0 + mk;) {  // runs of adjacent host slots
+  // one chunk's PCIe copies: runs of adjacent host slots among entries [i0, i0 + mk),
+  // layers [la, lb)
+  auto dma = [&](int32_t la, int32_t lb, int32_t i0, int32_t mk, uint8_t* buf) -> wind_status {
+    uint8_t* hplane0 = host->base + static_cast<int64_t>(la - host->desc.first_layer) * 2 * hpitch;
+    const size_t rows = static_cast<size_t>(2) * (lb - la);
+    for (int32_t j = i0; j < i0 + mk;) {
       int32_t r = 1;
       while (j + r < i0 + mk && hbt[j + r] == hbt[j] + r) ++r;
       uint8_t* hp = hplane0 + static_cast<int64_t>(hbt[j]) * C;
       uint8_t* sp = buf + static_cast<int64_t>(j - i0) * C;
-      WKV_CUDA(out ? cudaMemcpy2DAsync(hp, hpitch, sp, spitch, static_cast<size_t>(r * C), planes,
+      WKV_CUDA(out ? cudaMemcpy2DAsync(hp, hpitch, sp, spitch, static_cast<size_t>(r * C), rows,
                                        cudaMemcpyDeviceToHost, g.side)
-                   : cudaMemcpy2DAsync(sp, spitch, hp, hpitch, static_cast<size_t>(r * C), planes,
+                   : cudaMemcpy2DAsync(sp, spitch, hp, hpitch, static_cast<size_t>(r * C), rows,
                                        cudaMemcpyHostToDevice, g.side),
                "cudaMemcpy2DAsync(staged)");
       j += r;
     }
     return WIND_OK;
   };
-  const int32_t K = (it.n + m - 1) / m;
-  wind_status st;
+  const int32_t bchunks = (it.n + m - 1) / m;  // block chunks per layer group
+  const int32_t lgroups = (hi - lo + lpc - 1) / lpc;
+  const int32_t K = lgroups * bchunks;
   for (int32_t k = 0; k < K; ++k) {
-    const int32_t i0 = k * m, mk = std::min(m, it.n - i0), b = k & 1;
+    const int32_t la = lo + (k / bchunks) * lpc, lb = std::min(hi, la + lpc);
+    const int32_t i0 = (k % bchunks) * m, mk = std::min(m, it.n - i0), b = k & 1;
+    const bool layers_done = k % bchunks == bchunks - 1;  // last block chunk of [la, lb)
     stage.base = g.buf[b];
+    stage.desc.first_layer = la;
+    stage.desc.n_layers = lb - la;
+    stage.bytes = static_cast<size_t>(2 * (lb - la) * spitch);
     if (out) {
       if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(s, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
       OpItem gi{&stage, dev_bt + i0, g.iota, mk};
-      if ((st = run_op(dev, &gi, 1, lo, hi, s, HeadRange(), k == 0 ? &t_exposed : &t_hidden)) != WIND_OK)
+      if ((st = run_op(dev, &gi, 1, la, lb, s, HeadRange(), k == 0 ? &t_exposed : &t_hidden)) != WIND_OK)
         return st;
       WKV_CUDA(cudaEventRecord(g.ready[b], s), "cudaEventRecord(ready)");
       WKV_CUDA(cudaStreamWaitEvent(g.side, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
-      if ((st = dma(i0, mk, g.buf[b])) != WIND_OK) return st;
+      if ((st = dma(la, lb, i0, mk, g.buf[b])) != WIND_OK) return st;
+      if (layers_done && (st = flag_range(la, lb, g.side)) != WIND_OK) return st;
       WKV_CUDA(cudaEventRecord(g.freed[b], g.side), "cudaEventRecord(freed)");
     } else {
       if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(g.side, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
-      if ((st = dma(i0, mk, g.buf[b])) != WIND_OK) return st;
+      if ((st = dma(la, lb, i0, mk, g.buf[b])) != WIND_OK) return st;
       WKV_CUDA(cudaEventRecord(g.ready[b], g.side), "cudaEventRecord(ready)");
       WKV_CUDA(cudaStreamWaitEvent(s, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
       OpItem si{&shadow, g.iota, dev_bt + i0, mk};
-      if ((st = run_op(&stage, &si, 1, lo, hi, s, HeadRange(), k == K - 1 ? &t_exposed : &t_hidden)) != WIND_OK)
+      if ((st = run_op(&stage, &si, 1, la, lb, s, HeadRange(), k == K - 1 ? &t_exposed : &t_hidden)) != WIND_OK)
         return st;
+      if (layers_done && (st = flag_range(la, lb, s)) != WIND_OK) return st;
       WKV_CUDA(cudaEventRecord(g.freed[b], s), "cudaEventRecord(freed)");
     }
   }
-  if (out)  // join: the side stream's last copy (it runs its work in order)
+  if (out)  // join: the side stream's last copy and flags (it runs its work in order)
     WKV_CUDA(cudaStreamWaitEvent(s, g.freed[(K - 1) & 1], 0), "cudaStreamWaitEvent(join)");
-  // dst's layer flags: every layer once, after all chunks (system scope: a host pool's flags
-  // are read by the CPU; a device pool's by any stream)
-  Params fp;
-  memset(&fp, 0, sizeof fp);
-  fp.n_items = 1;
-  fp.items[0].flags = it.dst->flags;
-  fp.items[0].d_layers = it.dst->desc.n_layers;
-  fp.items[0].host_flags = it.dst->desc.loc == WIND_LOC_HOST;
-  fp.items[0].sys_scope = 1;
-  fp.sys_scope = 1;
-  WKV_CUDA(launch_flag_bump(fp, s), "flag kernel launch");
-  g_launches += 1;
   if (!capturing) {
     WKV_CUDA(cudaEventRecord(g.done, s), "cudaEventRecord(done)");
     g.has_done = true;

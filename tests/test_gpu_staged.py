@@ -4,9 +4,11 @@ device staging buffer, the copy engines over PCIe per run of adjacent host slots
 buffers pipelined on a side stream.  Every result is compared with the CPU oracle over
 the WHOLE host pool and device pool (untouched slots included), plus the layer flags.
 
-Chunking: the staging buffer holds m = max(32 MiB, 2 L C) // (2 (hi - lo) C) blocks, so
-C1 geometry (576 KiB per block) gives m = 56 and a 128-block swap runs 3 chunks with a
-ragged last one; a 64-layer, 288 KiB-chunk geometry gives m = 1 (one block per chunk).
+Chunking (layer-major): the staging buffer holds max(32 MiB, 2 L C) bytes; a chunk is as
+many whole layers of all n blocks as fit, else one layer of m = buffer // (2 C) blocks.
+C1 geometry with 128 blocks (6 MiB per layer) gives 3 chunks of 5, 5 and 2 layers; a
+2-layer, 288 KiB-chunk pool with 130 blocks gives 3 block chunks (56, 56, 18) per layer.
+dst's layer flags move as each layer's last chunk lands: one flag kernel per layer group.
 """
 import numpy as np
 import pytest
@@ -55,17 +57,23 @@ def htab(a) -> torch.Tensor:  # host-readable (pinned): selects the staged path
     return torch.as_tensor(np.asarray(a, np.int32)).pin_memory()
 
 
-def chunks(n: int, sh: KVShape, lo: int, hi: int, host_layers: int) -> int:
+def plan(n: int, sh: KVShape, lo: int, hi: int, host_layers: int):
+    """(chunks, layer groups) of the staged path (wind_kv.cpp staged_host_op)."""
     C = sh.n_kv_heads * sh.block_size * sh.head_dim * sh.elem_bytes
     buf = max(32 << 20, 2 * host_layers * C)
-    m = min(1 << 16, buf // (2 * C), buf // (2 * (hi - lo) * C))
-    return -(-n // m)
+    iota_n = min(1 << 16, buf // (2 * C))
+    if n <= iota_n and 2 * C * n <= buf:
+        lpc, m = min(hi - lo, buf // (2 * C * n)), n
+    else:
+        lpc, m = 1, min(iota_n, buf // (2 * C))
+    groups = -(-(hi - lo) // lpc)
+    return groups * -(-n // m), groups
 
 
 @pytest.mark.parametrize("host_tables", ["shuffled", "runs", "sequential"])
 def test_staged_round_trip_c1(host_tables):
-    """C1 geometry, 128 blocks -> 3 chunks (56, 56, 16): swap_out to host slots that are
-    fragmented / in runs / one run, then swap_in to DIFFERENT device slots."""
+    """C1 geometry, 128 blocks -> 3 layer-group chunks (5, 5, 2 layers): swap_out to host
+    slots that are fragmented / in runs / one run, then swap_in to DIFFERENT device slots."""
     case = migration_case("C1", scale=0.5)
     sh = case.shape
     n = case.n
@@ -82,12 +90,12 @@ def test_staged_round_trip_c1(host_tables):
     hbt = hbt.astype(np.int32)
     dev, d0 = pool(sh, case.nb_src, 1)
     host, h0 = pool(sh, nbh, 2, loc="host")
-    k = chunks(n, sh, 0, sh.n_layers, sh.n_layers)
-    assert k == 3
+    k, groups = plan(n, sh, 0, sh.n_layers, sh.n_layers)
+    assert (k, groups) == (3, 3)
     l0 = wk.launch_count()
     wk.swap_out(dev, dtab(case.src_bt), host, htab(hbt))
     torch.cuda.synchronize()
-    assert wk.launch_count() - l0 == k + 1  # k gathers + one flag kernel
+    assert wk.launch_count() - l0 == k + groups  # k gathers + one flag kernel per layer group
     want_h = h0.copy()
     assert O.swap_out(d0, geom(dev), case.src_bt, want_h, geom(host), hbt) == O.OK
     np.testing.assert_array_equal(host.tensor().numpy(), want_h)
@@ -105,26 +113,63 @@ def test_staged_round_trip_c1(host_tables):
     assert dev2.layer_ticket() == 1 and host.layer_ticket() == 1
 
 
-def test_staged_one_block_per_chunk():
-    """2 L C > 32 MiB: the buffer holds exactly one block of every layer (m = 1)."""
-    sh = KVShape("c3-64l", 64, 72, 128, 2)  # C = 288 KiB, 2 L C = 36 MiB -> buf 36 MiB, m = 1
-    n = 5
-    dev, d0 = pool(sh, 7, 4)
-    host, h0 = pool(sh, 6, 5, loc="host")
-    assert chunks(n, sh, 0, sh.n_layers, sh.n_layers) == 5
-    sbt = np.array([6, 0, 3, 2, 5], np.int32)
-    hbt = np.array([1, 2, 3, 0, 5], np.int32)
+def test_staged_block_chunks_within_a_layer():
+    """One layer of all blocks exceeds the buffer: each layer is split into block chunks
+    (56, 56, 18), layer-major; swap out and back in, byte-exact, flags once per layer."""
+    sh = KVShape("c3-2l", 2, 72, 128, 2)  # C = 288 KiB: 2 C n = 73 MiB per layer > 32 MiB
+    n = 130
+    assert plan(n, sh, 0, 2, 2) == (6, 2)
+    rng = np.random.default_rng(4)
+    dev, d0 = pool(sh, 140, 4)
+    host, h0 = pool(sh, 135, 5, loc="host")
+    sbt = rng.permutation(140)[:n].astype(np.int32)
+    hbt = rng.permutation(135)[:n].astype(np.int32)
+    l0 = wk.launch_count()
     wk.swap_out(dev, dtab(sbt), host, htab(hbt))
     torch.cuda.synchronize()
+    assert wk.launch_count() - l0 == 6 + 2
     want = h0.copy()
     assert O.swap_out(d0, geom(dev), sbt, want, geom(host), hbt) == O.OK
     np.testing.assert_array_equal(host.tensor().numpy(), want)
-    dev2, e0 = pool(sh, 9, 6)
-    dbt = np.array([8, 1, 0, 4, 7], np.int32)
+    dev2, e0 = pool(sh, 131, 6)
+    dbt = rng.permutation(131)[:n].astype(np.int32)
     wk.swap_in(host, htab(hbt), dev2, dtab(dbt))
     want2 = e0.copy()
     assert O.swap_in(want, geom(host), hbt, want2, geom(dev2), dbt) == O.OK
     np.testing.assert_array_equal(read(dev2), want2)
+    assert [dev2.layer_count(l) for l in range(2)] == [1, 1]
+
+
+def test_staged_swap_in_layer_flags_order_data():
+    """Per-layer streaming on the staged path: a consumer stream waits on each layer's flag
+    (wind_kv_layer_wait) and then snapshots that layer's K/V planes; every snapshot must
+    already hold the swapped-in bytes (flags are published after the layer's scatter)."""
+    case = migration_case("C2", scale=0.05)
+    sh = case.shape  # 40 layers, C = 160 KiB
+    n = case.n
+    dev, d0 = pool(sh, case.nb_src, 17)
+    host, _ = pool(sh, n, 18, loc="host")
+    hbt = np.arange(n, dtype=np.int32)
+    wk.swap_out(dev, dtab(case.src_bt), host, htab(hbt))
+    dev2, e0 = pool(sh, case.nb_dst, 19)
+    torch.cuda.synchronize()
+    want = e0.copy()
+    a = d0.reshape(sh.n_layers, 2, case.nb_src, -1)[:, :, case.src_bt]
+    want.reshape(sh.n_layers, 2, case.nb_dst, -1)[:, :, case.dst_bt] = a
+    plane = 2 * case.nb_dst * sh.chunk_bytes
+    s, cons = torch.cuda.Stream(DEV), torch.cuda.Stream(DEV)
+    snaps = torch.empty(sh.n_layers, plane, dtype=torch.uint8, device=DEV)
+    view = dev2.tensor()
+    for trial in range(3):
+        wk.swap_in(host, htab(hbt), dev2, dtab(case.dst_bt), stream=s)
+        t = dev2.layer_ticket()
+        with torch.cuda.stream(cons):
+            for l in range(sh.n_layers):
+                wk.layer_wait(dev2, l, t, stream=cons)
+                snaps[l].copy_(view[l * plane:(l + 1) * plane])
+        torch.cuda.synchronize()
+        np.testing.assert_array_equal(snaps.cpu().numpy().reshape(-1), want)
+        assert dev2.layer_count(0) == trial + 1
 
 
 @pytest.mark.parametrize("lo,hi", [(4, 10), (6, 7), (8, 10)])
