@@ -216,6 +216,13 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
     s = torch.cuda.Stream(device)
     hbm = peaks["hbm_gbs"]
 
+    # (0) C1 intra-device (BJ:configs[0], S§8(d) C1 (i)): migrate pool A -> pool B, and
+    #     compact pool A after a seeded half of its 8 requests is freed.  The working set
+    #     (2 x 144 MiB) is ~2.3 x L2, so the L2 is flushed (a READ of 2 x l2CacheSize:
+    #     clean lines, so no write-backs spill into the timed op) before every timed op,
+    #     outside its events.
+    out["c1_intra"] = run_c1_intra(wk, device, peaks, reps=20, warmup=warmup)
+
     # (1) C2 sequential tables (long runs: the coalescing / TMA best case)
     case = migration_case("C2", variant="sequential")
     sh = case.shape
@@ -345,6 +352,50 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
     out["next3_backup_reshard"] = run_next3(wk, device, peaks)
     torch.cuda.empty_cache()
     return out
+
+
+def run_c1_intra(wk, device, peaks, reps=20, warmup=3) -> dict:
+    import torch
+    from windgen import migration_case, live_mask_after_free, request_lengths, blocks_for_tokens
+    dev = torch.device("cuda", device)
+    s = torch.cuda.Stream(device)
+    hbm = peaks["hbm_gbs"]
+    case = migration_case("C1")
+    sh = case.shape
+    a = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
+    b = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag)
+    sbt, dbt = torch.as_tensor(case.src_bt, device=dev), torch.as_tensor(case.dst_bt, device=dev)
+    l2 = int(getattr(torch.cuda.get_device_properties(device), "L2_cache_size", 0) or (126 << 20))
+    flush = torch.ones(2 * l2 // 4, dtype=torch.int32, device=dev)
+
+    def timed(fn):
+        for _ in range(warmup):
+            fn()
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(reps)]
+        torch.cuda.synchronize()
+        with torch.cuda.stream(s):
+            for e0, e1 in ev:
+                flush.sum(dtype=torch.int64)  # evicts both pools' lines (untimed)
+                e0.record(s)
+                fn()
+                e1.record(s)
+        torch.cuda.synchronize()
+        return float(np.median([e0.elapsed_time(e1) for e0, e1 in ev]))
+    pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
+    ms = timed(lambda: wk.migrate(a, sbt, b, dbt, stream=s))
+    res = {"migrate_gbs": round(pb / ms / 1e6, 1), "migrate_hbm_frac": round(2 * pb / ms / 1e6 / hbm, 3),
+           "migrate_ms": round(ms, 4), "payload_mib": round(pb / (1 << 20), 1),
+           "l2_flush_read_bytes_before_each_op": int(flush.numel() * 4)}
+    reqb = blocks_for_tokens(request_lengths("C1"), sh.block_size)
+    live, _ = live_mask_after_free(case.nb_src, reqb, 0.5, 4001)
+    csrc, cdst = wk.plan_compact(live)
+    ts, td = torch.as_tensor(csrc, device=dev), torch.as_tensor(cdst, device=dev)
+    pc = payload_bytes(len(csrc), sh.n_layers, sh.chunk_bytes)
+    ms = timed(lambda: wk.compact(a, ts, td, stream=s))
+    res.update({"compact_moves": int(len(csrc)), "compact_gbs": round(pc / ms / 1e6, 1),
+                "compact_hbm_frac": round(2 * pc / ms / 1e6 / hbm, 3), "compact_ms": round(ms, 4)})
+    del a, b, flush
+    return res
 
 
 def run_next3(wk, device, peaks, steps=10, warmup=3) -> dict:

@@ -30,6 +30,7 @@ fn = {"interference": lambda: bench.run_interference(wk, 0, peaks),
       "interference_configs": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=30,
                                                              configs=small_footprint),
       "pressure": lambda: bench.run_pressure(wk, 0),
+      "c1_intra": lambda: bench.run_c1_intra(wk, 0, peaks),
       "interference_rw": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=40, configs=[
           (n, c) for n, c in [
               ("control_no_migration", {**wk.get_tuning(wk.PATH_INTRA), "null_feeder": True}),
