@@ -56,7 +56,7 @@ class ClockSampler:
 
     Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
          "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
-         "clocks_event_reasons.sw_power_cap")
+         "clocks_event_reasons.sw_power_cap,power.draw")
 
     def __init__(self, device: int):
         self.device = device
@@ -76,7 +76,7 @@ class ClockSampler:
 
     def _read(self):
         for line in self.proc.stdout:
-            self.lines.append(line.strip())
+            self.lines.append((time.time(), line.strip()))  # host arrival time (~ms)
 
     def __exit__(self, *a):
         if self.proc:
@@ -86,10 +86,14 @@ class ClockSampler:
             except Exception:
                 self.proc.kill()
 
-    def summary(self) -> dict:
-        sm, mx, reasons = [], None, set()
+    def summary(self, t0: float = 0.0, t1: float = float("inf")) -> dict:
+        """Median SM clock and power, and every throttle reason seen, over the samples that
+        arrived in host time [t0, t1] (default: all)."""
+        sm, pw, mx, reasons = [], [], None, set()
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
+        for t, ln in list(self.lines):
+            if not t0 <= t <= t1:
+                continue
             f = [x.strip() for x in ln.split(",")]
             if len(f) < 6:
                 continue
@@ -101,8 +105,13 @@ class ClockSampler:
             for n, v in zip(names, f[2:6]):
                 if v.lower().startswith("active"):
                     reasons.add(n)
+            try:
+                pw.append(float(f[6]))
+            except (IndexError, ValueError):
+                pass
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "reasons": sorted(reasons), "samples": len(sm),
+                "power_w": round(float(np.median(pw)), 1) if pw else None}
 
 
 # ----------------------------------------------------------------------- helpers
@@ -802,6 +811,8 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
          ("swap_in_staged", {"op": "swap_in", **saved_host, "kernel": wk.KERNEL_STAGED})])
     rounds, n_round = 3, max(10, n_victim_steps // 2)
     part = {}  # SM partition (green contexts): victim graph on the compute SMs
+    clk = ClockSampler(device).__enter__()  # SM clock / power per phase (power-cap effects)
+    time.sleep(1.0)  # nvidia-smi start-up
 
     def partitioned(min_sms):
         if min_sms not in part:
@@ -846,6 +857,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         t_mig = time_device(one_op, 2, 3, mig_s) / 2
         full_alone = []
         alone_all, with_all, covered = [], [], True
+        win_alone, win_with = [], []
         # `rounds` interleaved pairs (victim alone, then victim + migration): the alone
         # reference is always adjacent in time (removes clock / power drift).  A feeder
         # thread keeps exactly one migration op in flight on the low-priority stream for the
@@ -857,8 +869,10 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
                 ev = victim_run(n_round)
                 torch.cuda.synchronize()
                 full_alone += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
+            ta0 = time.time()
             ev = victim_run(n_round, vic_g, vic_s)
             torch.cuda.synchronize()
+            win_alone.append((ta0, time.time()))
             alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
             stop, started, n_ops = threading.Event(), threading.Event(), [0]
 
@@ -875,8 +889,10 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             th = threading.Thread(target=feeder, daemon=True)
             th.start()
             started.wait()
+            tw0 = time.time()
             ev = victim_run(n_round, vic_g, vic_s)
             torch.cuda.synchronize()
+            win_with.append((tw0, time.time()))
             stop.set()
             th.join()
             covered &= th is not None and n_ops[0] >= 1
@@ -893,11 +909,26 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             "victim_ms_with_migration": round(t_with, 3),
             "slowdown": round(t_with / t_ref - 1.0, 4),
             "migration_covered_all_victim_steps": bool(covered)}
+
+        def phase(wins):
+            sm, pw, rs = [], [], set()
+            for a_, b_ in wins:
+                c_ = clk.summary(a_, b_)
+                if c_["sm_mhz"] is not None:
+                    sm.append(c_["sm_mhz"])
+                if c_["power_w"] is not None:
+                    pw.append(c_["power_w"])
+                rs |= set(c_["reasons"])
+            return {"sm_mhz": float(np.median(sm)) if sm else None,
+                    "power_w": round(float(np.median(pw)), 1) if pw else None, "reasons": sorted(rs)}
+        res[name]["clocks_alone"] = phase(win_alone)
+        res[name]["clocks_with_migration"] = phase(win_with)
         if min_sms:
             t_full = float(np.median(full_alone))
             res[name].update({"partition_sms_migration": P.sms_migration, "partition_sms_compute": P.sms_compute,
                               "victim_ms_alone_whole_gpu": round(t_full, 3),
                               "slowdown_vs_whole_gpu": round(t_with / t_full - 1.0, 4)})
+    clk.__exit__()
     wk.set_tuning(wk.PATH_INTRA, **saved)
     wk.set_tuning(wk.PATH_HOST, **saved_host)
     torch.cuda.synchronize()
