@@ -15,3 +15,11 @@ timeout -s KILL 900 compute-sanitizer --tool racecheck --print-limit 20 python -
   "tests/test_gpu_parity.py::test_migrate_c1_all_kernels" "tests/test_gpu_parity.py::test_run_coalescing_across_warp_windows" \
   > gpurun_out/sanitize_racecheck_tests.txt 2>&1
 echo "racecheck tests rc=$? $(tail -2 gpurun_out/sanitize_racecheck_tests.txt | head -1)"
+# the staged copy-engine swap path (events, side stream, staging buffers)
+timeout -s KILL 900 compute-sanitizer --tool memcheck --print-limit 20 python -m pytest -q -x \
+  "tests/test_gpu_staged.py" > gpurun_out/sanitize_memcheck_staged.txt 2>&1
+echo "memcheck staged rc=$? $(tail -2 gpurun_out/sanitize_memcheck_staged.txt | head -1)"
+timeout -s KILL 900 compute-sanitizer --tool racecheck --print-limit 20 python -m pytest -q -x \
+  "tests/test_gpu_staged.py::test_staged_round_trip_c1" "tests/test_gpu_staged.py::test_staged_block_chunks_within_a_layer" \
+  > gpurun_out/sanitize_racecheck_staged.txt 2>&1
+echo "racecheck staged rc=$? $(tail -2 gpurun_out/sanitize_racecheck_staged.txt | head -1)"
