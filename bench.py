@@ -1057,6 +1057,32 @@ def run_gpu(args) -> None:
         if role != "decode":
             wk.migrate(src, sbt, dst, dbt, layer_lo=lo, layer_hi=hi, stream=stream)
 
+    # N > 1: the peer-path kernel is chosen on the real link before the timed steps (round 1
+    # never had two GPUs in one call, so the default was never measured over NVLink 5):
+    # every candidate runs the same op for 3 steps (max over ranks), the fastest becomes the
+    # PEER tuning for the headline.  Reported as `peer_autotune` in the line.
+    peer_tune = None
+    if world > 1:
+        cands = [("simt_96ctas", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=32768, stages=6,
+                                       max_ctas=96)),
+                 ("simt_4x148", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768, stages=6)),
+                 ("tma_148", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, store_lag=2)),
+                 ("tma_64", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, store_lag=2,
+                                 max_ctas=64)),
+                 ("tma_32", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, store_lag=2,
+                                 max_ctas=32))]
+        try:
+            rates = {}
+            for name, cfg in cands:
+                wk.set_tuning(wk.PATH_PEER, **cfg)
+                ms_alt, = parallel.max_over_ranks([time_device(step, 3, 3, stream, barrier) / 3])
+                rates[name] = round(pb / ms_alt / 1e6, 1)
+            best = max(rates, key=rates.get)
+            wk.set_tuning(wk.PATH_PEER, **dict(cands)[best])
+            peer_tune = {"chosen": best, "gbs_per_pair": rates}
+        except Exception as e:  # noqa: BLE001 — reported; the library default stays
+            peer_tune = {"error": f"{type(e).__name__}: {e}"[:300]}
+            print(f"[bench rank {rank}] peer autotune failed: {peer_tune['error']}", file=sys.stderr, flush=True)
     torch.cuda.synchronize()
     launches0 = wk.launch_count()
     step_ms: list = []
@@ -1087,27 +1113,11 @@ def run_gpu(args) -> None:
     n_movers = parallel.movers(world)
     total_bytes = pb * n_movers
     a2a = None
-    peer_alt = None
     scen_error = None
     if world > 1 and args.scenarios:
         # The multi-GPU scenarios never ran on more than one GPU in round 1 (one GPU per
         # gpurun call): a failure there is reported in the line, never loses the headline.
         try:
-            # the peer-path kernel choice: time the alternatives on the real link (same op,
-            # 3 steps each, max over ranks)
-            peer_alt = {}
-            saved = wk.get_tuning(wk.PATH_PEER)
-            for name, cfg in [("simt_96ctas", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=32768,
-                                                    max_ctas=96)),
-                              ("simt_4x148", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768)),
-                              ("tma_148", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4,
-                                               store_lag=2)),
-                              ("tma_32", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4,
-                                              store_lag=2, max_ctas=32))]:
-                wk.set_tuning(wk.PATH_PEER, **cfg)
-                ms_alt, = parallel.max_over_ranks([time_device(step, 3, 3, stream, barrier) / 3])
-                peer_alt[name] = round(pb / ms_alt / 1e6, 1)
-            wk.set_tuning(wk.PATH_PEER, **saved)
             torch.cuda.synchronize()
             del src, dst
             torch.cuda.empty_cache()
@@ -1136,8 +1146,10 @@ def run_gpu(args) -> None:
                     "frac_of_nominal_900": round(kernel_gbs / 900.0, 4),
                     "per_launch_bytes": pb}
         extra["roofline"] = roof
+        if peer_tune is not None:
+            extra["peer_autotune"] = peer_tune
         if a2a is not None or scen_error is not None:
-            extra["scenarios"] = {"c5_all_to_all": a2a, "peer_kernel_gbs_per_pair": peer_alt}
+            extra["scenarios"] = {"c5_all_to_all": a2a}
             if scen_error is not None:
                 extra["scenarios"]["error"] = scen_error
         if world == 1 and not args.no_cpu_baseline:
