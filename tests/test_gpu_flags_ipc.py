@@ -162,9 +162,9 @@ def test_ipc_push_and_pull_between_processes():
         side = pattern_pool(sh, 70, 9, 4)
         sb2 = rng.permutation(120)[:40].astype(np.int32)
         db2 = rng.permutation(70)[:40].astype(np.int32)
-        wk.migrate_batch(src, [(remote, torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)),
-                               (side, torch.as_tensor(sb2, device=DEV), torch.as_tensor(db2, device=DEV))],
-                         1, 4, stream=s)
+        # tables are borrowed until the ops on `s` complete: keep them referenced
+        tabs = [torch.as_tensor(x, device=DEV) for x in (sbt, dbt, sb2, db2, dbt[:10])]
+        wk.migrate_batch(src, [(remote, tabs[0], tabs[1]), (side, tabs[2], tabs[3])], 1, 4, stream=s)
         t = remote.layer_ticket()
         for l in range(4):
             wk.layer_wait(remote, l, t, stream=s)
@@ -173,8 +173,8 @@ def test_ipc_push_and_pull_between_processes():
         # pull: remote -> a local pool
         back = pattern_pool(sh, 60, 9, 3)
         pb = np.arange(10, dtype=np.int32)
-        wk.migrate(remote, torch.as_tensor(dbt[:10], device=DEV), back, torch.as_tensor(pb, device=DEV),
-                   stream=s)
+        tabs.append(torch.as_tensor(pb, device=DEV))
+        wk.migrate(remote, tabs[4], back, tabs[5], stream=s)
         s.synchronize()
         q_in.put("done")
         got, counts, _ = q_out.get(timeout=300)
@@ -223,8 +223,8 @@ def test_full_size_c2_parity_every_chunk(variant):
     src = pattern_pool(sh, case.nb_src, case.content_seed, case.src_tag)
     dst = pattern_pool(sh, case.nb_dst, case.content_seed, case.dst_tag)
     s = torch.cuda.Stream(DEV)
-    wk.migrate(src, torch.as_tensor(case.src_bt, device=DEV), dst, torch.as_tensor(case.dst_bt, device=DEV),
-               stream=s)
+    ts, td = torch.as_tensor(case.src_bt, device=DEV), torch.as_tensor(case.dst_bt, device=DEV)
+    wk.migrate(src, ts, dst, td, stream=s)  # tables borrowed until the op completes
     s.synchronize()
     gs, gd = geom(src), geom(dst)
     from_src, off = O.expected_origin(gs, case.src_bt, gd, case.dst_bt, 0, sh.n_layers)

@@ -49,8 +49,24 @@ def read(p: wk.Pool) -> np.ndarray:
     return p.tensor().cpu().numpy().copy()
 
 
+_KEEP: list = []  # block tables are BORROWED until their op completes (wind_kv.h)
+
+
+@pytest.fixture(autouse=True)
+def keep_tables_alive():
+    yield
+    for d in range(torch.cuda.device_count()):
+        torch.cuda.synchronize(d)
+    _KEEP.clear()
+
+
 def tab(a, device: int) -> torch.Tensor:
-    return torch.as_tensor(np.asarray(a, np.int32), device=torch.device("cuda", device))
+    """A device table that stays alive until the test ends: the ops run on side streams, so a
+    temporary freed after the call could be reused by the caching allocator (on the default
+    stream) while the kernel still reads it."""
+    t = torch.as_tensor(np.asarray(a, np.int32), device=torch.device("cuda", device))
+    _KEEP.append(t)
+    return t
 
 
 def test_push_then_pull_across_devices():

@@ -160,8 +160,9 @@ def test_staged_swap_in_layer_flags_order_data():
     s, cons = torch.cuda.Stream(DEV), torch.cuda.Stream(DEV)
     snaps = torch.empty(sh.n_layers, plane, dtype=torch.uint8, device=DEV)
     view = dev2.tensor()
+    h_t, d_t = htab(hbt), dtab(case.dst_bt)  # borrowed until the ops complete
     for trial in range(3):
-        wk.swap_in(host, htab(hbt), dev2, dtab(case.dst_bt), stream=s)
+        wk.swap_in(host, h_t, dev2, d_t, stream=s)
         t = dev2.layer_ticket()
         with torch.cuda.stream(cons):
             for l in range(sh.n_layers):
