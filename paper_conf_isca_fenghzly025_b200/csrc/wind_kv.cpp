@@ -8,6 +8,7 @@
 #include <stdarg.h>
 #include <stdint.h>
 #include <stdio.h>
+#include <stdlib.h>
 #include <string.h>
 #include <dlfcn.h>
 #include <unistd.h>
@@ -152,6 +153,15 @@ wind_kv_tuning g_tune[3] = {
 //  - staged gather / scatter chunks hidden behind PCIe copies: ~768 KiB in flight keeps
 //    them ahead of PCIe (56-57 / 55 GB/s) with 4-6 % victim cost (1.5 MiB+: no faster).
 constexpr int64_t kHostToHostInFlight = 384 << 10;
+
+// WIND_KV_BLOCKED_DEALING=0 turns the small-op contiguous dealing off (A/B measurements).
+bool blocked_dealing_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("WIND_KV_BLOCKED_DEALING");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
 constexpr int kHostCtasFromHost = 8;
 constexpr int64_t kStagedInFlight = 768 << 10;
 
@@ -1067,6 +1077,12 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   if (t.rate_mbps > 0 && t.max_ctas == 0)
     grid = std::min<int64_t>(grid, std::max<int64_t>(1, (t.rate_mbps + kCtaMBps - 1) / kCtaMBps));
   grid = std::max<int64_t>(1, std::min<int64_t>(grid, p.total_units));
+  // Work dealing.  Grid-stride (all CTAs sweep the layers together: each layer completes
+  // early, A5 streaming) unless a plane has fewer units than the grid: then every CTA
+  // would cross a layer boundary at almost every unit, and each crossing waits for its
+  // older stores to be fully written before the arrival — a latency chain that dominates
+  // small ops.  Those get contiguous unit ranges per CTA (a handful of crossings each).
+  p.blocked = (p.units_per_plane < grid && t.rate_mbps == 0 && blocked_dealing_enabled()) ? 1 : 0;
   // rate limit: each of the `grid` CTAs gets rate / grid; ns per payload byte per CTA
   p.ns_per_byte = t.rate_mbps > 0 ? static_cast<float>(grid * 1e3 / t.rate_mbps) : 0.f;
   cudaError_t e = launch_copy(p, kernel, static_cast<int>(grid), s);

@@ -58,6 +58,8 @@ struct Params {
   int32_t stages;             // TMA ring depth
   int32_t stage_bytes;        // TMA stage size
   int32_t sys_scope;          // any item has sys_scope
+  int32_t blocked;            // 1: CTA c takes the contiguous unit range [c*per, (c+1)*per)
+                              // (small ops: fewer layer crossings per CTA); 0: grid-stride
   int32_t fan;                // > 1: read-once fan-out — every item shares items[0]'s source
                               // table and units; each staged unit is stored to all `fan`
                               // destinations (TMA kernel only; 1 otherwise)

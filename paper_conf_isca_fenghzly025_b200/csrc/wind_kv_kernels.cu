@@ -18,12 +18,15 @@
 // so all CTAs sweep the layers together and a layer completes early (A5 streaming).
 //
 // Layer completion (A5).  When a CTA leaves layer l (its next unit is in a later layer, or
-// it is done) it makes its stores of l complete and visible, then adds 1 to this op's
-// arrival counter for l; the CTA that brings the counter to gridDim.x publishes
-// dst.layer_done[l] += 1 behind a release fence — GPU scope when the data and the flags
-// stay on this GPU, system scope for a peer (NVLink) or host destination — and resets the
-// counter for the next op using the slot.  The TMA consumer defers the arrival until `lag`
-// newer store groups are in flight, so the store pipeline never drains at a layer boundary.
+// it is done) it makes its stores of l complete and visible, then adds the number of l's
+// units it moved to this op's arrival counter for l; the CTA that brings the counter to
+// the layer's unit total (2 planes x units_per_plane) publishes dst.layer_done[l] += 1
+// behind a release fence — GPU scope when the data and the flags stay on this GPU, system
+// scope for a peer (NVLink) or host destination — and resets the counter for the next op
+// using the slot.  A CTA arrives only on layers it touched (a small op's CTAs touch one or
+// two), so an op costs one counter atomic per (CTA, touched layer).  The TMA consumer
+// defers the arrival until `lag` newer store groups are in flight, so the store pipeline
+// never drains at a layer boundary.
 //
 // Kernels.
 //   tma_copy_kernel  (K2): 2 warps per CTA.  Warp 0 = producer: decodes units and issues
@@ -351,40 +354,37 @@ __device__ __forceinline__ void bulk_wait_done_n(int n) {
   }
 }
 
-// Arrive on layers [from, to) (global ids) of this op; the last CTA publishes.  Caller has
-// made this CTA's stores of those layers complete and ordered before this call.  The
-// counter atomics of a range are issued 8 at a time (independent round trips in flight).
-// Scope: when data and flags stay on this GPU (p.sys_scope == 0) every observer — the
-// consumer stream's wait, the kernels it releases, another process's CTAs on this device —
-// reads through this GPU's L2, so GPU-scope fences suffice; a fence.acq_rel.sys costs
-// ~1 us and, issued per layer, cost a 32-layer op ~50 us.
-__device__ void arrive_layers(const Params& p, int32_t from, int32_t to) {
-  if (from >= to) return;
+// Arrive on global layer `layer` with the `cnt` units of it this CTA moved; the arrival
+// that completes the layer's 2 x units_per_plane units publishes.  Caller has made this
+// CTA's stores of those units complete and ordered before this call.  Scope: when data and
+// flags stay on this GPU (p.sys_scope == 0) every observer — the consumer stream's wait,
+// the kernels it releases, another process's CTAs on this device — reads through this
+// GPU's L2, so GPU-scope fences suffice; a fence.acq_rel.sys costs ~1 us.
+__device__ void arrive_layer(const Params& p, int32_t layer, uint32_t cnt) {
+  if (cnt == 0) return;
   if (p.sys_scope)
     fence_sys();
   else
     fence_gpu();
-  for (int32_t l0 = from; l0 < to; l0 += 8) {
-    uint32_t old[8];
-#pragma unroll
-    for (int k = 0; k < 8; ++k)
-      if (l0 + k < to) old[k] = atomicAdd(p.counters + (l0 + k - p.layer_lo), 1u);
-    uint32_t last = 0;  // layers of this batch whose last arrival is this CTA's
-#pragma unroll
-    for (int k = 0; k < 8; ++k)
-      if (l0 + k < to && old[k] == gridDim.x - 1) last |= 1u << k;
-    if (!last) continue;
-    if (p.sys_scope)  // one release fence for every flag published below
-      fence_sys();
-    else
-      fence_gpu();
-    for (uint32_t m = last; m; m &= m - 1) {
-      const int32_t l = l0 + __ffs(m) - 1;
-      for (int j = 0; j < p.n_items; ++j)
-        bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (l - p.layer_lo), p.items[j]);
-      *reinterpret_cast<volatile uint32_t*>(p.counters + (l - p.layer_lo)) = 0u;  // slot reusable
-    }
-  }
+  uint32_t* c = p.counters + (layer - p.layer_lo);
+  const uint32_t total = 2u * static_cast<uint32_t>(p.units_per_plane);
+  if (atomicAdd(c, cnt) + cnt != total) return;
+  if (p.sys_scope)  // acquire the other arrivals, release the flags below
+    fence_sys();
+  else
+    fence_gpu();
+  for (int j = 0; j < p.n_items; ++j)
+    bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (layer - p.layer_lo), p.items[j]);
+  *reinterpret_cast<volatile uint32_t*>(c) = 0u;  // slot reusable
+}
+
+// Debug pools whose device table check fired: nothing is copied, but every layer flag of
+// the op still moves once (a consumer waiting on a ticket must not hang).
+__device__ void publish_aborted(const Params& p) {
+  fence_sys();
+  for (int32_t l = p.layer_lo; l < p.layer_lo + p.n_layers; ++l)
+    for (int j = 0; j < p.n_items; ++j)
+      bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (l - p.layer_lo), p.items[j]);
 }
 
 // ------------------------------------------------------------------- K2: TMA staged
@@ -410,16 +410,27 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
   }
   __syncthreads();
   if (blockIdx.x == 0 && threadIdx.x == 33) publish_untouched_layers(p);  // an idle consumer lane
+  if (p.abort_word && *reinterpret_cast<const volatile int32_t*>(p.abort_word)) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) publish_aborted(p);
+    return;
+  }
 
   if (warp == 0) {  // ------------------------------------------------ producer warp
     const uint64_t pol = ef ? evict_first_policy() : 0;
-    const int64_t total = (p.abort_word && *p.abort_word) ? 0 : p.total_units;
+    const int64_t total = p.total_units;
+    int64_t u0 = blockIdx.x, ustep = gridDim.x, uend = total;
+    if (p.blocked) {  // contiguous range: the CTA crosses few layer boundaries
+      const int64_t per = (p.total_units + gridDim.x - 1) / gridDim.x;
+      u0 = blockIdx.x * per;
+      ustep = 1;
+      uend = u0 + per < total ? u0 + per : total;
+    }
     Pacer pacer;
     int it = 0;
-    for (int64_t u = blockIdx.x;; u += gridDim.x, ++it) {
+    for (int64_t u = u0;; u += ustep, ++it) {
       const int st = it % S;
       if (it >= S) mbar_wait(&empty[st], ((it / S) & 1) ^ 1);
-      if (u >= total) {
+      if (u >= uend) {
         if (lane == 0) desc[st].nseg = -1;
         mbar_arrive(&full[st]);
         break;
@@ -448,13 +459,15 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
     // the producer's load lookahead)
     const int lag = p.store_lag > 0 ? p.store_lag : (S / 2 > 0 ? S / 2 : 1);
     // Layer arrivals without draining the store pipeline: when unit `it` opens a later
-    // layer, the stores of layers [cur, layer) are the bulk groups < it.  The arrival is
+    // layer, the stores of the layer just left are the bulk groups < it.  The arrival is
     // deferred until `lag` newer groups have been committed; then a full wait_group<lag>
     // (instead of this iteration's .read wait) makes exactly those groups complete.  A
     // second boundary while one is pending (< lag units per layer) resolves the first one
     // on the spot with a shallower wait.
-    int32_t cur = p.layer_lo;  // layers < cur have been arrived on by this CTA
-    int32_t pend_to = -1;      // pending arrival on [cur, pend_to) once groups < pend_it are done
+    int32_t cur = -1;          // layer of the units being stored, and how many of them
+    uint32_t cur_cnt = 0;
+    int32_t pend = -1;         // pending arrival on layer `pend` (pend_cnt units) once the
+    uint32_t pend_cnt = 0;     // groups < pend_it are done
     int pend_it = 0;
     for (int it = 0;; ++it) {
       const int st = it % S;
@@ -462,16 +475,19 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
       const int nseg = desc[st].nseg;
       if (nseg < 0) break;
       const int32_t layer = p.layer_lo + desc[st].plane / 2;
-      if (layer > (pend_to >= 0 ? pend_to : cur)) {  // this CTA is done with layers < layer
-        if (pend_to >= 0) {
+      if (cur >= 0 && layer != cur) {  // this CTA is done with layer `cur`
+        if (pend >= 0) {
           bulk_wait_done_n(it - pend_it);  // the it - pend_it groups >= pend_it may stay pending
           fence_async_global();
-          arrive_layers(p, cur, pend_to);
-          cur = pend_to;
+          arrive_layer(p, pend, pend_cnt);
         }
-        pend_to = layer;
+        pend = cur;
+        pend_cnt = cur_cnt;
         pend_it = it;
+        cur_cnt = 0;
       }
+      cur = layer;
+      ++cur_cnt;
       const uint8_t* sbuf = buf + static_cast<size_t>(st) * SB;
       for (int k = 0; k < nseg; ++k) {
         const Seg& g = desc[st].segs[k];
@@ -483,12 +499,11 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
           bulk_store(desc[st].fdst[f - 1][k], sbuf + g.soff, g.len, ef, pol);
         }
       bulk_commit();
-      if (pend_to >= 0 && it - pend_it + 1 >= lag) {
+      if (pend >= 0 && it - pend_it + 1 >= lag) {
         bulk_wait_done_n(it - pend_it + 1);  // groups < pend_it complete (and <= it - lag read)
         fence_async_global();
-        arrive_layers(p, cur, pend_to);
-        cur = pend_to;
-        pend_to = -1;
+        arrive_layer(p, pend, pend_cnt);
+        pend = -1;
       } else {
         bulk_wait_read_n(lag);  // stores of units <= it - lag have read their stage
       }
@@ -496,7 +511,8 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
     }
     bulk_wait_all();
     fence_async_global();
-    arrive_layers(p, cur, p.layer_lo + p.n_layers);
+    if (pend >= 0) arrive_layer(p, pend, pend_cnt);
+    if (cur >= 0) arrive_layer(p, cur, cur_cnt);
   }
 }
 
@@ -512,10 +528,22 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
   const bool ef = p.evict_first != 0;
   const uint64_t pol = ef ? evict_first_policy() : 0;
   if (blockIdx.x == 0 && tid == 32) publish_untouched_layers(p);  // not the decoding warp
-  int32_t cur = p.layer_lo;
-  const int64_t total = (p.abort_word && *p.abort_word) ? 0 : p.total_units;
+  if (p.abort_word && *reinterpret_cast<const volatile int32_t*>(p.abort_word)) {
+    if (blockIdx.x == 0 && tid == 0) publish_aborted(p);
+    return;
+  }
+  int32_t cur = -1;  // layer of the units being copied, and how many of them
+  uint32_t cur_cnt = 0;
+  const int64_t total = p.total_units;
+  int64_t u0 = blockIdx.x, ustep = gridDim.x, uend = total;
+  if (p.blocked) {
+    const int64_t per = (p.total_units + gridDim.x - 1) / gridDim.x;
+    u0 = blockIdx.x * per;
+    ustep = 1;
+    uend = u0 + per < total ? u0 + per : total;
+  }
   Pacer pacer;
-  for (int64_t u = blockIdx.x; u < total; u += gridDim.x) {
+  for (int64_t u = u0; u < uend; u += ustep) {
     if (tid < 32) {
       int32_t plane;
       uint32_t bytes;
@@ -528,10 +556,12 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
     }
     __syncthreads();
     const int32_t layer = p.layer_lo + s_plane / 2;
-    if (layer > cur) {  // uniform: every thread of the CTA left layers [cur, layer)
-      if (tid == 0) arrive_layers(p, cur, layer);
-      cur = layer;
+    if (cur >= 0 && layer != cur) {  // uniform: every thread of the CTA left layer `cur`
+      if (tid == 0) arrive_layer(p, cur, cur_cnt);
+      cur_cnt = 0;
     }
+    cur = layer;
+    ++cur_cnt;
     const int nseg = s_nseg;
     for (int k = 0; k < nseg; ++k) {
       const int4* s = reinterpret_cast<const int4*>(segs[k].src);
@@ -558,7 +588,7 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
     }
     __syncthreads();  // all stores of this unit issued; segs may be overwritten
   }
-  if (tid == 0) arrive_layers(p, cur, p.layer_lo + p.n_layers);
+  if (tid == 0 && cur >= 0) arrive_layer(p, cur, cur_cnt);
 }
 
 // ------------------------------------------------- copy-engine path: flag publication
