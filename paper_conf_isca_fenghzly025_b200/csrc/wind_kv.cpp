@@ -165,19 +165,60 @@ bool blocked_dealing_enabled() {
 constexpr int kHostCtasFromHost = 8;
 constexpr int64_t kStagedInFlight = 768 << 10;
 
-// Bytes one work unit covers for copies of CP bytes per block with units of at most `unit`
-// bytes (the decomposition run_op gives the kernels).
-int64_t work_unit_bytes(int64_t CP, int64_t unit) {
-  if (CP >= unit) {
-    const int64_t parts = (CP + unit - 1) / unit;
-    return ((CP + parts - 1) / parts + 15) / 16 * 16;
+// Work decomposition and TMA ring of an op copying CP bytes per (layer, kv, block) under a
+// tuning (stage_bytes, stages, store_lag).  A chunk larger than a stage is split in `parts`
+// equal 16-B-multiple pieces; smaller chunks are grouped `group` per unit (a warp-window of
+// table entries).  For the TMA kernel the group is ROUNDED to the nearest count (C4's
+// 32 KiB chunks in 48 KiB stages: 2 per unit, not 1 — per-unit overheads bound a CTA, and
+// 32 KiB units ran C4 at 0.93 of HBM, 64 KiB units at 0.96) and the ring re-shaped to keep
+// stages x stage_bytes bytes in flight (at least 3 stages, within shared memory), the
+// store lag the same fraction of the ring.
+struct Ring {
+  int32_t parts = 1, part_bytes = 0, group = 1;  // decomposition
+  int64_t unit = 0;                              // bytes per work unit
+  int32_t stages = 0, stage_bytes = 0, lag = 0;  // TMA ring (the tuning's when unchanged)
+};
+
+Ring plan_ring(int64_t CP, const wind_kv_tuning& t, bool tma) {
+  Ring r;
+  r.stages = t.stages;
+  r.stage_bytes = t.stage_bytes;
+  r.lag = t.store_lag;
+  const int64_t SB = t.stage_bytes;
+  if (CP >= SB) {
+    r.parts = static_cast<int32_t>((CP + SB - 1) / SB);
+    r.part_bytes = static_cast<int32_t>((((CP + r.parts - 1) / r.parts) + 15) / 16 * 16);
+    r.unit = r.part_bytes;
+    return r;
   }
-  return std::min<int64_t>(kMaxSegs, unit / CP) * CP;
+  r.part_bytes = static_cast<int32_t>(CP);
+  int64_t g = std::min<int64_t>(kMaxSegs, SB / CP);
+  r.group = static_cast<int32_t>(g);
+  r.unit = g * CP;
+  if (!tma) return r;
+  const int64_t budget = static_cast<int64_t>(t.stages) * SB;
+  const int64_t g2 = std::min<int64_t>(kMaxSegs, (SB + CP / 2) / CP);  // nearest
+  const int64_t u2 = g2 * CP;
+  if (u2 == SB) return r;
+  const int64_t s2 = std::min<int64_t>(16, std::max<int64_t>(3, budget / u2));
+  if (tma_smem_bytes(static_cast<int>(s2), static_cast<int>(u2)) > 227 * 1024) return r;
+  r.group = static_cast<int32_t>(g2);
+  r.unit = u2;
+  r.stages = static_cast<int32_t>(s2);
+  r.stage_bytes = static_cast<int32_t>(u2);
+  if (t.store_lag > 0)
+    r.lag = static_cast<int32_t>(std::min<int64_t>(s2 - 1, std::max<int64_t>(1, (t.store_lag * s2) / t.stages)));
+  return r;
 }
 
-int ctas_for_in_flight(int64_t target, int stages, int64_t unit_bytes) {
-  const int64_t per_cta = std::max<int64_t>(1, static_cast<int64_t>(stages) * unit_bytes);
+int ctas_for_in_flight(int64_t target, const Ring& r) {
+  const int64_t per_cta = std::max<int64_t>(1, static_cast<int64_t>(r.stages) * r.unit);
   return static_cast<int>(std::max<int64_t>(1, (target + per_cta - 1) / per_cta));
+}
+
+int staged_hidden_ctas(int64_t chunk) {  // the staged path's hidden chunks: kStagedInFlight
+  const wind_kv_tuning tg = {kTma, 1, 49152, 4, 0, 0, 2, 0};
+  return ctas_for_in_flight(kStagedInFlight, plan_ring(chunk, tg, true));
 }
 
 }  // namespace
@@ -957,7 +998,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     if (staged)  // hidden chunks run the staged kernel tuning (4 x 48 KiB stages)
       return staged_host_op(src, items[0], lo, hi, s,
                             t.max_ctas > 0 ? t.max_ctas
-                                           : ctas_for_in_flight(kStagedInFlight, 4, work_unit_bytes(src->chunk, 49152)));
+                                           : staged_hidden_ctas(src->chunk));
     if (t.kernel == kStaged)
       return fail(WIND_ERR_UNSUPPORTED, "staged path needs one item, whole chunks, no rate limit, a "
                   "host-readable host table and host-pool staging on device %d", exec);
@@ -986,27 +1027,21 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   const int64_t CS = src->chunk;
   const int64_t tile = static_cast<int64_t>(src->desc.block_size) * src->desc.head_dim * src->desc.elem_bytes;
   const int64_t CP = hr.n < 0 ? CS : hr.n * tile;  // bytes copied per (layer, kv, block)
-  const int64_t unit = t.stage_bytes;
+  const Ring ring = plan_ring(CP, t, kernel == kTma);
   p.s_chunk = CS;
   p.copy = CP;
-  if (CP >= unit) {
-    p.parts = static_cast<int32_t>((CP + unit - 1) / unit);
-    p.part_bytes = static_cast<int32_t>((((CP + p.parts - 1) / p.parts) + 15) / 16 * 16);
-    p.group = 1;
-  } else {
-    p.parts = 1;
-    p.part_bytes = static_cast<int32_t>(CP);
-    p.group = static_cast<int32_t>(std::min<int64_t>(kMaxSegs, unit / CP));
-  }
+  p.parts = ring.parts;
+  p.part_bytes = ring.part_bytes;
+  p.group = ring.group;
   p.layer_lo = lo;
   p.n_layers = hi - lo;
   p.src_plane0 = src->base + static_cast<int64_t>(lo - src->desc.first_layer) * 2 * src->desc.n_blocks * CS +
                  (hr.n < 0 ? 0 : hr.src_lo * tile);
   p.s_plane_stride = static_cast<int64_t>(src->desc.n_blocks) * CS;
   p.evict_first = t.evict_first;
-  p.store_lag = t.store_lag;
-  p.stages = t.stages;
-  p.stage_bytes = t.stage_bytes;
+  p.store_lag = ring.lag;
+  p.stages = ring.stages;
+  p.stage_bytes = ring.stage_bytes;
   int32_t base_units = 0;
   int ni = 0;
   for (int j = 0; j < n_items; ++j) {
@@ -1067,9 +1102,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   else if (path == WIND_PATH_HOST) {
     bool to_host = false;  // any store into host memory: the backpressure-prone direction
     for (int j = 0; j < n_items; ++j) to_host = to_host || items[j].dst->desc.loc == WIND_LOC_HOST;
-    grid = std::min<int64_t>(grid, to_host ? ctas_for_in_flight(kHostToHostInFlight, t.stages,
-                                                                work_unit_bytes(CP, t.stage_bytes))
-                                           : kHostCtasFromHost);
+    grid = std::min<int64_t>(grid, to_host ? ctas_for_in_flight(kHostToHostInFlight, ring) : kHostCtasFromHost);
   }
   // A rate-limited op holds as few SMs as can sustain the rate (one CTA moves ~38 GB/s of
   // payload intra-device): the SMs a migration occupies cost a co-running HBM-bound decode
