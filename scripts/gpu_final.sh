@@ -9,3 +9,8 @@ timeout -s KILL 1500 ncu --metrics gpu__time_duration.sum --clock-control none -
    --log-file gpurun_out/launches_final.csv python bench.py --steps 5 --warmup 3 --no-cpu-baseline \
    > gpurun_out/launches_bench_final.json 2>&1
 echo "launches rc=$?"
+# full section set on the headline launch (application replay: the pools are ~95 GiB)
+timeout -s KILL 1500 ncu --set full --clock-control none --import-source on --replay-mode application \
+   -k regex:tma_copy -s 3 -c 1 -o gpurun_out/prof_tma_c2_final \
+   python bench.py --steps 1 --warmup 3 --no-scenarios --no-cpu-baseline > gpurun_out/prof_bench_final.json 2>&1
+echo "full rc=$?"
