@@ -161,7 +161,11 @@ wind_status wind_kv_pool_import(const wind_kv_ipc_handle* handle, int32_t local_
  *     polls a LOCAL op's flags must order its reads through CUDA events / streams; flags of
  *     dst layers outside
  *     [lo, hi) are incremented at the start of the op, so "flag >= ticket" is meaningful
- *     for every layer.  Layers are processed in ascending order.
+ *     for every layer.  Layers are processed in ascending order: every CTA walks
+ *     its work units layer-major, so on ops with at least as many work units per (layer,
+ *     K|V) plane as CTAs the flags complete layer by layer while the op runs; smaller ops
+ *     give each CTA a contiguous unit range and their layers complete near the op's end,
+ *     in no guaranteed order (a flag still never moves before its layer's bytes).
  *   n_blocks == 0 or layer_lo == layer_hi: WIND_OK, nothing enqueued, no ticket (R19). */
 wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind_kv_pool* dst,
                             const int32_t* dst_bt, int32_t n_blocks, int32_t layer_lo,
