@@ -11,7 +11,7 @@
 namespace wkv {
 
 // Ring of per-op, per-layer CTA-arrival counters on each executing device (A5).  An op
-// takes slot (seq % kCounterSlots); the last CTA to arrive on a layer resets the counter,
+// takes slot (seq % kCounterSlots); the arrival completing a layer's units resets the counter,
 // so a slot is reusable as soon as the op that used it has finished.
 constexpr int kCounterSlots = 512;  // 2 MiB per device; ops in flight CONCURRENTLY (across streams) <= 512
 constexpr int kMaxSegs = 32;  // segments (runs) per work unit = one warp's table window
