@@ -858,6 +858,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         full_alone = []
         alone_all, with_all, covered = [], [], True
         win_alone, win_with = [], []
+        co_bytes, co_secs = 0, 0.0
         # `rounds` interleaved pairs (victim alone, then victim + migration): the alone
         # reference is always adjacent in time (removes clock / power drift).  A feeder
         # thread keeps exactly one migration op in flight on the low-priority stream for the
@@ -875,6 +876,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             win_alone.append((ta0, time.time()))
             alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
             stop, started, n_ops = threading.Event(), threading.Event(), [0]
+            done_t: list = []  # host time of each op completion (migration rate while co-running)
 
             def feeder():
                 while not stop.is_set():
@@ -885,6 +887,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
                     one_op()
                     started.set()
                     mig_s.synchronize()
+                    done_t.append(time.time())
                     n_ops[0] += 1
             th = threading.Thread(target=feeder, daemon=True)
             th.start()
@@ -892,9 +895,14 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             tw0 = time.time()
             ev = victim_run(n_round, vic_g, vic_s)
             torch.cuda.synchronize()
-            win_with.append((tw0, time.time()))
+            tw1 = time.time()
+            win_with.append((tw0, tw1))
             stop.set()
             th.join()
+            ts = [t for t in done_t if tw0 <= t <= tw1]
+            if len(ts) >= 2:
+                co_bytes += op_bytes * (len(ts) - 1)
+                co_secs += ts[-1] - ts[0]
             covered &= th is not None and n_ops[0] >= 1
             with_all += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
             alone_all += alone
@@ -908,6 +916,9 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             "victim_ms_alone_adjacent": round(t_ref, 3),
             "victim_ms_with_migration": round(t_with, 3),
             "slowdown": round(t_with / t_ref - 1.0, 4),
+            # the migration's own rate WHILE the victim runs (ops completed inside the victim
+            # window; None when fewer than 2 completed there, e.g. slow rate-limited ops)
+            "migration_gbs_during": round(co_bytes / co_secs / 1e9, 1) if co_secs > 0 else None,
             "migration_covered_all_victim_steps": bool(covered)}
 
         def phase(wins):

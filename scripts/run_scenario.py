@@ -75,6 +75,16 @@ fn = {"interference": lambda: bench.run_interference(wk, 0, peaks),
               ("staged_out_h4_b", "swap_out", dict(kernel=4, max_ctas=4)),
               ("sm_out_tma2_b", "swap_out", dict(kernel=1, max_ctas=2)),
           ]]),
+      "interference_ce": lambda: bench.run_interference(wk, 0, peaks, n_victim_steps=40, configs=[
+          (n, {**wk.get_tuning(wk.PATH_INTRA), **c}) for n, c in [
+              ("ce_rate50", dict(kernel=3, rate_mbps=50000)),
+              ("ce_rate150", dict(kernel=3, rate_mbps=150000)),
+              ("ce_rate300", dict(kernel=3, rate_mbps=300000)),
+              ("ce_rate450", dict(kernel=3, rate_mbps=450000)),
+              ("ce_rate600", dict(kernel=3, rate_mbps=600000)),
+              ("ce_unlimited", dict(kernel=3, rate_mbps=0)),
+              ("ce_rate300_b", dict(kernel=3, rate_mbps=300000)),
+              ("ce_rate150_b", dict(kernel=3, rate_mbps=150000))]]),
       "policy": lambda: bench.run_policy_profile(wk, 0),
       "stall_free": lambda: bench.run_stall_free(wk, 0),
       "handoff": lambda: bench.run_handoff(wk, 0),
