@@ -312,7 +312,11 @@ typedef struct {
                        back PCIe writes up into the GPU's memory system: 1.5 MiB in flight
                        slowed a co-running decode kernel by 73 %, 384 KiB by 2 %, same
                        52 GB/s), 8 CTAs from host memory; staged path: hidden gather /
-                       scatter chunks with ~768 KiB in flight (4-6 CTAs) */
+                       scatter chunks with ~768 KiB in flight (4-6 CTAs).
+                       PEER path: the same backpressure is expected when SM stores outrun
+                       NVLink; for pushes next to latency-sensitive work on the SOURCE GPU,
+                       cap the CTAs (or rate_mbps) so the link is not oversubscribed
+                       (not measurable with one GPU per round-1 call) */
   int32_t evict_first; /* 1 = L2 evict-first policy on the copy's loads and stores */
   int32_t store_lag;   /* TMA: stores allowed in flight per CTA (0 = stages / 2) */
   int32_t rate_mbps;   /* payload rate limit of one op in MB/s (0 = unlimited): bounds the
