@@ -281,23 +281,10 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
     del src, dst
 
     # (3) C5 compaction on GPU 0's share of the skewed placement (A7)
-    sh5 = SHAPES["C5"]
-    lens = request_lengths("C5")
-    place = skewed_placement(lens.size, 8, 4005)
-    reqb = blocks_for_tokens(lens[place == 0], 16)
-    nb = math.ceil(int(reqb.sum()) * 1.1)
-    live, _ = live_mask_after_free(nb, reqb, 0.5, 4006)
-    csrc, cdst = wk.plan_compact(live)
-    pool = make_pool(wk, sh5, nb, device, 3005, 1)
-    ts, td = torch.as_tensor(csrc, device=dev), torch.as_tensor(cdst, device=dev)
-    pb = payload_bytes(len(csrc), sh5.n_layers, sh5.chunk_bytes)
-    # compaction is idempotent under repetition only for the first run; moving the same
-    # pairs again re-copies identical bytes (same traffic), which is what is timed
-    ms = time_device(lambda: wk.compact(pool, ts, td, stream=s), 5 * steps, warmup, s) / (5 * steps)
+    pb, ms, moves, pool_gib = run_c5_compaction(wk, device, 0, 5 * steps, warmup)
     gbs = pb / ms / 1e6
     out["c5_compact"] = {"gbs": round(gbs, 1), "hbm_frac": round(2 * gbs / hbm, 3), "ms": round(ms, 3),
-                         "moves": int(len(csrc)), "pool_gib": round(pool.nbytes / GiB, 2)}
-    del pool
+                         "moves": moves, "pool_gib": pool_gib}
 
     # (4) C1 host swap round trip over PCIe (A6): swap_out then swap_in at other slots
     case = migration_case("C1")
@@ -361,6 +348,31 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
     out["next3_backup_reshard"] = run_next3(wk, device, peaks)
     torch.cuda.empty_cache()
     return out
+
+
+def run_c5_compaction(wk, device, gpu_index, steps, warmup, barrier=None):
+    """A7 on GPU `gpu_index`'s share of C5's skewed placement over 8 GPUs: free a seeded
+    half of its requests, plan_compact, compact.  Returns (payload bytes, ms per op, moves,
+    pool GiB).  Repeating the op re-copies identical bytes (same traffic): that is timed."""
+    import torch
+    from windgen import (SHAPES, live_mask_after_free, skewed_placement, request_lengths,
+                         blocks_for_tokens)
+    dev = torch.device("cuda", device)
+    s = torch.cuda.Stream(device)
+    sh5 = SHAPES["C5"]
+    lens = request_lengths("C5")
+    place = skewed_placement(lens.size, 8, 4005)
+    reqb = blocks_for_tokens(lens[place == gpu_index % 8], 16)
+    nb = math.ceil(int(reqb.sum()) * 1.1)
+    live, _ = live_mask_after_free(nb, reqb, 0.5, 4006 + gpu_index)
+    csrc, cdst = wk.plan_compact(live)
+    pool = make_pool(wk, sh5, nb, device, 3005, 1 + gpu_index)
+    ts, td = torch.as_tensor(csrc, device=dev), torch.as_tensor(cdst, device=dev)
+    pb = payload_bytes(len(csrc), sh5.n_layers, sh5.chunk_bytes)
+    ms = time_device(lambda: wk.compact(pool, ts, td, stream=s), steps, warmup, s, barrier) / steps
+    gib = round(pool.nbytes / GiB, 2)
+    del pool
+    return pb, ms, int(len(csrc)), gib
 
 
 def run_c1_intra(wk, device, peaks, reps=20, warmup=3) -> dict:
@@ -1124,6 +1136,7 @@ def run_gpu(args) -> None:
     n_movers = parallel.movers(world)
     total_bytes = pb * n_movers
     a2a = None
+    compaction = None
     scen_error = None
     if world > 1 and args.scenarios:
         # The multi-GPU scenarios never ran on more than one GPU in round 1 (one GPU per
@@ -1133,6 +1146,14 @@ def run_gpu(args) -> None:
             del src, dst
             torch.cuda.empty_cache()
             a2a = run_all_to_all(wk, rank, world, local, peaks, scale=args.a2a_scale)
+            # intra-device work at N GPUs (A7): every rank compacts its own share of C5 at
+            # the same time (GPU g holds placement share g mod 8); aggregate = sum / max time
+            pbc, msc, _, _ = run_c5_compaction(wk, local, rank, 10, 3, barrier=dist.barrier)
+            tot_b = torch.tensor([float(pbc)], dtype=torch.float64)
+            dist.all_reduce(tot_b)
+            ms_c, = parallel.max_over_ranks([msc])
+            compaction = {"aggregate_gbs": round(float(tot_b.item()) / ms_c / 1e6, 1), "ms_max": round(ms_c, 3),
+                          "hbm_frac_per_gpu": round(2 * float(tot_b.item()) / world / ms_c / 1e6 / peaks["hbm_gbs"], 3)}
         except Exception as e:  # noqa: BLE001 — reported, not swallowed
             scen_error = f"{type(e).__name__}: {e}"[:400]
             print(f"[bench rank {rank}] multi-GPU scenario failed: {scen_error}", file=sys.stderr, flush=True)
@@ -1160,7 +1181,7 @@ def run_gpu(args) -> None:
         if peer_tune is not None:
             extra["peer_autotune"] = peer_tune
         if a2a is not None or scen_error is not None:
-            extra["scenarios"] = {"c5_all_to_all": a2a}
+            extra["scenarios"] = {"c5_all_to_all": a2a, "c5_compaction_all_ranks": compaction}
             if scen_error is not None:
                 extra["scenarios"]["error"] = scen_error
         if world == 1 and not args.no_cpu_baseline:
