@@ -1004,6 +1004,8 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
                   "host-readable host table and host-pool staging on device %d", exec);
   }
   const int kernel = t.kernel == kAuto ? (path == WIND_PATH_PEER ? kSimt : kTma) : t.kernel;
+  if (kernel == kStaged)
+    return fail(WIND_ERR_UNSUPPORTED, "kernel 4 (staged copy engines) moves host pools only");
   // Read-once fan-out (backups; NEXT-3): when every item of a batch walks the SAME
   // source table (same pointer and length), the TMA kernel stages each source unit once and
   // stores it to every destination — (1 + k) x payload of DRAM traffic instead of 2k x.
@@ -1341,6 +1343,8 @@ extern "C" wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t)
   std::lock_guard<std::mutex> lk(g_tune_mu);
   wind_kv_tuning n = g_tune[path];
   if (t->kernel < 0 || t->kernel > 4) return fail(WIND_ERR_INVALID_ARG, "kernel must be 0 .. 4");
+  if (t->kernel == kStaged && path != WIND_PATH_HOST)
+    return fail(WIND_ERR_INVALID_ARG, "kernel 4 (staged copy engines) is a HOST-path kernel");
   n.kernel = t->kernel;
   if (t->ctas_per_sm) n.ctas_per_sm = t->ctas_per_sm;
   if (t->stage_bytes) n.stage_bytes = t->stage_bytes;

@@ -101,8 +101,16 @@ def test_tuning_roundtrip_and_bounds():
     assert e.value.status == -1
     with pytest.raises(wk.WindKVError):
         wk.set_tuning(wk.PATH_PEER, stage_bytes=131072, stages=4)  # > 227 KiB smem
+    with pytest.raises(wk.WindKVError) as e:  # staged copy engines: HOST path only
+        wk.set_tuning(wk.PATH_PEER, kernel=wk.KERNEL_STAGED)
+    assert e.value.status == -1
     wk.set_tuning(wk.PATH_PEER, **{k: v for k, v in old.items()})
     assert wk.get_tuning(wk.PATH_PEER) == old
+    old_h = wk.get_tuning(wk.PATH_HOST)
+    wk.set_tuning(wk.PATH_HOST, **{**old_h, "kernel": wk.KERNEL_STAGED})
+    assert wk.get_tuning(wk.PATH_HOST)["kernel"] == wk.KERNEL_STAGED
+    wk.set_tuning(wk.PATH_HOST, **old_h)
+    assert wk.get_tuning(wk.PATH_HOST) == old_h
 
 
 def test_null_arguments_fail_cleanly_without_gpu():

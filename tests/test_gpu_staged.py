@@ -271,6 +271,12 @@ def test_staged_errors():
     assert wk.launch_count() == l0 and host.layer_ticket() == 0
     torch.cuda.synchronize()
     np.testing.assert_array_equal(host.tensor().numpy(), h0)
+    # kernel 4 on device -> device: UNSUPPORTED (never silently another kernel)
+    other, _ = pool(sh, case.nb_src, 17)
+    with pytest.raises(wk.WindKVError) as e:
+        wk.migrate_ex(dev, dtab(case.src_bt), other, dtab(case.src_bt),
+                      wk.tuning(kernel=wk.KERNEL_STAGED))
+    assert e.value.status == -10
     # the auto choice falls back to the SM kernel for a device-resident host table
     wk.set_tuning(wk.PATH_HOST, kernel=wk.KERNEL_AUTO)
     l0 = wk.launch_count()
