@@ -183,7 +183,8 @@ wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind
  *     dst's layer flags move as each layer's last chunk lands (layer_wait works as for
  *     migrate).  host_bt is READ ON THE CPU at enqueue (entries out of range: BLOCK_RANGE,
  *     nothing enqueued).  Staged ops on one host pool serialise on its buffers
- *     automatically outside graph capture (inside a capture, order them yourself).
+ *     automatically outside graph capture (inside a capture, order them yourself); they
+ *     must be enqueued by one host thread at a time (the pool's events are reused).
  *   - otherwise SM / TMA stores to and loads from mapped pinned memory over PCIe, per-layer
  *     flags as in migrate.
  * A host pool's layer flags live in mapped host memory and are updated without PCIe
