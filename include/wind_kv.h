@@ -62,6 +62,8 @@ typedef enum { WIND_LOC_DEVICE = 0, WIND_LOC_HOST = 1 /* pinned, mapped, portabl
 
 /* Pool flags. */
 #define WIND_POOL_DEBUG 0x1u /* ops into/out of this pool also run a device table check */
+#define WIND_POOL_NO_STAGING 0x2u /* host pools: no copy-engine staging (saves 2 x max(32 MiB,
+                                     2 L C) of device memory; swaps use the SM kernels) */
 
 /* Pool descriptor.  Layout (reading R2): [L][2][NB][H][bs][d] elements of
  * elem_bytes, layer-major with K/V planes; chunk (layer l, kv, block b) is the C =

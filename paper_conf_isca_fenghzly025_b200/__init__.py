@@ -36,6 +36,7 @@ STATUS = {
 OK = 0
 LOC_DEVICE, LOC_HOST = 0, 1
 POOL_DEBUG = 0x1
+POOL_NO_STAGING = 0x2
 PATH_INTRA, PATH_PEER, PATH_HOST = 0, 1, 2
 KERNEL_AUTO, KERNEL_TMA, KERNEL_SIMT, KERNEL_COPY_ENGINE, KERNEL_STAGED = 0, 1, 2, 3, 4
 IPC_HANDLE_BYTES = 512
@@ -197,11 +198,11 @@ class Pool:
     def __init__(self, n_layers: int, n_kv_heads: int, head_dim: int, block_size: int,
                  elem_bytes: int, n_blocks: int, *, loc: str = "device", device: int = 0,
                  first_layer: int = 0, debug: bool = False, external_base: Optional[int] = None,
-                 _handle: Optional[int] = None):
+                 staging: bool = True, _handle: Optional[int] = None):
         if _handle is None:
             d = PoolDesc(first_layer, n_layers, n_kv_heads, head_dim, block_size, elem_bytes,
                          n_blocks, LOC_HOST if loc == "host" else LOC_DEVICE, device,
-                         POOL_DEBUG if debug else 0)
+                         (POOL_DEBUG if debug else 0) | (0 if staging else POOL_NO_STAGING))
             h = ct.c_void_p()
             _check(lib().wind_kv_pool_create(ct.byref(d), external_base, ct.byref(h)))
             _handle = h.value

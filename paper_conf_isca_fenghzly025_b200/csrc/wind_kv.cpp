@@ -412,7 +412,7 @@ extern "C" wind_status wind_kv_pool_create(const wind_kv_pool_desc* desc, void* 
     return fail(WIND_ERR_OOM, "layer flag allocation failed: %s", cudaGetErrorString(e));
   }
   p->owns_flags = true;
-  if (desc->loc == WIND_LOC_HOST) staging_init(p, desc->device);
+  if (desc->loc == WIND_LOC_HOST && !(desc->flags & WIND_POOL_NO_STAGING)) staging_init(p, desc->device);
   *out = p;
   return WIND_OK;
 }

@@ -283,3 +283,24 @@ def test_staged_errors():
     wk.swap_out(dev, dtab(case.src_bt), host, dtab(np.arange(case.n)))
     torch.cuda.synchronize()
     assert wk.launch_count() - l0 == 1
+
+
+def test_no_staging_flag_uses_the_sm_path():
+    """WIND_POOL_NO_STAGING: the host pool gets no device staging, so even a host-readable
+    table takes the SM kernel over mapped memory (one launch); byte-exact either way."""
+    case = migration_case("C1", scale=0.25)
+    sh = case.shape
+    dev, d0 = pool(sh, case.nb_src, 20)
+    host = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, case.n,
+                   loc="host", staging=False)
+    h0 = np.random.default_rng(21).integers(0, 256, host.nbytes, dtype=np.uint8)
+    host.tensor().copy_(torch.from_numpy(h0))
+    hbt = np.random.default_rng(22).permutation(case.n).astype(np.int32)
+    st, ht = dtab(case.src_bt), htab(hbt)
+    l0 = wk.launch_count()
+    wk.swap_out(dev, st, host, ht)
+    torch.cuda.synchronize()
+    assert wk.launch_count() - l0 == 1
+    want = h0.copy()
+    assert O.swap_out(d0, geom(dev), case.src_bt, want, geom(host), hbt) == O.OK
+    np.testing.assert_array_equal(host.tensor().numpy(), want)
