@@ -1058,7 +1058,7 @@ def run_gpu(args) -> None:
     peaks = load_peaks()
 
     from paper_conf_isca_fenghzly025_b200 import parallel
-    case = migration_case(args.config, variant=args.variant)
+    case = migration_case(args.config, variant=args.variant, seed_offset=args.seed)
     sh = case.shape
     role, partner = parallel.pair_role(rank, world)
     src = dst = None
@@ -1204,7 +1204,7 @@ def run_gpu(args) -> None:
                        "payload_gib_per_pair": round(pb / GiB, 3),
                        "placement": "same GPU" if world == 1 else "pairs 2k->2k+1 over NVLink peer stores",
                        "l2": "inputs >> 126 MB L2 (no flush needed)",
-                       "parallelism": f"{n_movers} independent mover(s)"},
+                       "parallelism": f"{n_movers} independent mover(s)", "seed_offset": args.seed},
             "e2e": {"value": round(e2e_value, 2), "unit": "GB/s",
                     "h2d_bytes_per_step": int(8 * case.n), "d2h_bytes_per_step": int(4 * sh.n_layers)},
             "gpu_launches": int(launches),
@@ -1243,7 +1243,7 @@ def run_reference(args) -> None:
         return
     import oracle as O
     from windgen import migration_case
-    case = migration_case(args.config, variant=args.variant)
+    case = migration_case(args.config, variant=args.variant, seed_offset=args.seed)
     sh = case.shape
     n = min(64, case.n)  # bounded sample per step
     nb = math.ceil(1.1 * n)
@@ -1282,6 +1282,8 @@ def main():
     ap.add_argument("--impl", default="wind_kv", choices=["wind_kv", "reference"])
     ap.add_argument("--config", default="C2")
     ap.add_argument("--variant", default="shuffled", choices=["shuffled", "sequential"])
+    ap.add_argument("--seed", type=int, default=0,
+                    help="offset of the config's length / slot / content seeds (0 = the S§8(d) seeds)")
     ap.add_argument("--scenarios", dest="scenarios", action="store_true", default=True)
     ap.add_argument("--no-scenarios", dest="scenarios", action="store_false")
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -135,11 +135,12 @@ SHAPES = {
 }
 
 
-def request_lengths(cfg: str, scale: float = 1.0) -> np.ndarray:
+def request_lengths(cfg: str, scale: float = 1.0, seed_offset: int = 0) -> np.ndarray:
     """Token lengths of the requests each config migrates.  ``scale`` < 1
-    shrinks the request COUNT (not the distribution) for small parity cases."""
+    shrinks the request COUNT (not the distribution) for small parity cases;
+    ``seed_offset`` shifts the config's seed (bench --seed)."""
     k = int(cfg[1])
-    seed = 1000 + k
+    seed = 1000 + k + seed_offset
     if cfg == "C1":
         n = max(1, round(8 * scale))
         return np.full(n, 512, dtype=np.int64)
@@ -205,13 +206,15 @@ class MigrationCase:
 
 def migration_case(cfg: str, variant: str = "shuffled", scale: float = 1.0,
                    lengths: np.ndarray | None = None, shape: KVShape | None = None,
-                   occupied_frac: float = 0.30) -> MigrationCase:
+                   occupied_frac: float = 0.30, seed_offset: int = 0) -> MigrationCase:
     """The common generator of SURVEY §8(d): NB_src = ceil(1.1*n); sources = first n of
     a seeded permutation (shuffled) or 0..n-1 (sequential); the destination pool has a
-    seeded 30 % of slots pre-occupied and takes the lowest free slots (A10)."""
-    k = int(cfg[1])
+    seeded 30 % of slots pre-occupied and takes the lowest free slots (A10).
+    ``seed_offset`` shifts every seed of the config (len / slot / content; bench --seed)."""
+    k = int(cfg[1]) + seed_offset
     shape = shape or SHAPES[cfg]
-    lens = request_lengths(cfg, scale) if lengths is None else np.asarray(lengths, np.int64)
+    lens = (request_lengths(cfg, scale, seed_offset) if lengths is None
+            else np.asarray(lengths, np.int64))
     req_blocks = blocks_for_tokens(lens, shape.block_size)
     n = int(req_blocks.sum())
     nb_src = max(1, math.ceil(1.1 * n))
