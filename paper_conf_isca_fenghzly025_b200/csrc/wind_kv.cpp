@@ -251,7 +251,7 @@ struct wind_kv_pool {
     int32_t* iota = nullptr;          // 0, 1, ..., iota_n - 1: the staging side's block table
     int32_t iota_n = 0;
     uint32_t* dummy_flags = nullptr;  // layer flags of the internal gather / scatter ops
-    cudaStream_t side = nullptr;
+    cudaStream_t side[2] = {nullptr, nullptr};  // DMA streams (swap out uses both)
     cudaEvent_t fork = nullptr, done = nullptr, ready[2] = {nullptr, nullptr},
                 freed[2] = {nullptr, nullptr};
     bool has_done = false;            // `done` marks the end of the last uncaptured staged op
@@ -296,7 +296,8 @@ void staging_free(wind_kv_pool::Staging& g) {
   if (g.dummy_flags) cudaFree(g.dummy_flags);
   if (g.fork) cudaEventDestroy(g.fork);
   if (g.done) cudaEventDestroy(g.done);
-  if (g.side) cudaStreamDestroy(g.side);
+  for (int b = 0; b < 2; ++b)
+    if (g.side[b]) cudaStreamDestroy(g.side[b]);
   cudaGetLastError();
   g = wind_kv_pool::Staging();
 }
@@ -324,7 +325,8 @@ void staging_init(wind_kv_pool* p, int dev) {
             cudaMemcpy(g.iota, iota.data(), sizeof(int32_t) * g.iota_n, cudaMemcpyHostToDevice) == cudaSuccess &&
             cudaMalloc(&g.dummy_flags, sizeof(uint32_t) * WIND_KV_MAX_LAYERS) == cudaSuccess &&
             cudaMemset(g.dummy_flags, 0, sizeof(uint32_t) * WIND_KV_MAX_LAYERS) == cudaSuccess &&
-            cudaStreamCreateWithFlags(&g.side, cudaStreamNonBlocking) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&g.side[0], cudaStreamNonBlocking) == cudaSuccess &&
+            cudaStreamCreateWithFlags(&g.side[1], cudaStreamNonBlocking) == cudaSuccess &&
             cudaEventCreateWithFlags(&g.fork, cudaEventDisableTiming) == cudaSuccess &&
             cudaEventCreateWithFlags(&g.done, cudaEventDisableTiming) == cudaSuccess;
   for (int b = 0; ok && b < 2; ++b)
@@ -871,11 +873,19 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
   const int32_t f0 = it.dst->desc.first_layer, f1 = f0 + it.dst->desc.n_layers;
   if ((st = flag_range(f0, lo, s)) != WIND_OK) return st;
   if ((st = flag_range(hi, f1, s)) != WIND_OK) return st;
+  const int32_t bchunks = (it.n + m - 1) / m;  // block chunks per layer group
+  const int32_t lgroups = (hi - lo + lpc - 1) / lpc;
+  const int32_t K = lgroups * bchunks;
+  // DMA streams: a swap-out alternates chunks over two (two device-to-host copies in flight
+  // drive PCIe ~3.5 % harder than one: 55.9 vs 54.0 GB/s, scripts/ce_parallel_probe.py);
+  // host-to-device gains nothing from a second stream, so a swap-in uses one
+  const int nside = (out && K >= 2) ? 2 : 1;
   WKV_CUDA(cudaEventRecord(g.fork, s), "cudaEventRecord(fork)");
-  WKV_CUDA(cudaStreamWaitEvent(g.side, g.fork, 0), "cudaStreamWaitEvent(fork)");
+  for (int q = 0; q < nside; ++q)
+    WKV_CUDA(cudaStreamWaitEvent(g.side[q], g.fork, 0), "cudaStreamWaitEvent(fork)");
   // one chunk's PCIe copies: runs of adjacent host slots among entries [i0, i0 + mk),
-  // layers [la, lb)
-  auto dma = [&](int32_t la, int32_t lb, int32_t i0, int32_t mk, uint8_t* buf) -> wind_status {
+  // layers [la, lb), on DMA stream `ds`
+  auto dma = [&](int32_t la, int32_t lb, int32_t i0, int32_t mk, uint8_t* buf, cudaStream_t ds) -> wind_status {
     uint8_t* hplane0 = host->base + static_cast<int64_t>(la - host->desc.first_layer) * 2 * hpitch;
     const size_t rows = static_cast<size_t>(2) * (lb - la);
     for (int32_t j = i0; j < i0 + mk;) {
@@ -884,17 +894,14 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
       uint8_t* hp = hplane0 + static_cast<int64_t>(hbt[j]) * C;
       uint8_t* sp = buf + static_cast<int64_t>(j - i0) * C;
       WKV_CUDA(out ? cudaMemcpy2DAsync(hp, hpitch, sp, spitch, static_cast<size_t>(r * C), rows,
-                                       cudaMemcpyDeviceToHost, g.side)
+                                       cudaMemcpyDeviceToHost, ds)
                    : cudaMemcpy2DAsync(sp, spitch, hp, hpitch, static_cast<size_t>(r * C), rows,
-                                       cudaMemcpyHostToDevice, g.side),
+                                       cudaMemcpyHostToDevice, ds),
                "cudaMemcpy2DAsync(staged)");
       j += r;
     }
     return WIND_OK;
   };
-  const int32_t bchunks = (it.n + m - 1) / m;  // block chunks per layer group
-  const int32_t lgroups = (hi - lo + lpc - 1) / lpc;
-  const int32_t K = lgroups * bchunks;
   for (int32_t k = 0; k < K; ++k) {
     const int32_t la = lo + (k / bchunks) * lpc, lb = std::min(hi, la + lpc);
     const int32_t i0 = (k % bchunks) * m, mk = std::min(m, it.n - i0), b = k & 1;
@@ -908,15 +915,20 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
       OpItem gi{&stage, dev_bt + i0, g.iota, mk};
       if ((st = run_op(dev, &gi, 1, la, lb, s, HeadRange(), k == 0 ? &t_exposed : &t_hidden)) != WIND_OK)
         return st;
+      cudaStream_t ds = g.side[b % nside];
       WKV_CUDA(cudaEventRecord(g.ready[b], s), "cudaEventRecord(ready)");
-      WKV_CUDA(cudaStreamWaitEvent(g.side, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
-      if ((st = dma(la, lb, i0, mk, g.buf[b])) != WIND_OK) return st;
-      if (layers_done && (st = flag_range(la, lb, g.side)) != WIND_OK) return st;
-      WKV_CUDA(cudaEventRecord(g.freed[b], g.side), "cudaEventRecord(freed)");
+      WKV_CUDA(cudaStreamWaitEvent(ds, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
+      if ((st = dma(la, lb, i0, mk, g.buf[b], ds)) != WIND_OK) return st;
+      if (layers_done) {
+        // the layers' earlier chunks may have gone over the other DMA stream
+        if (nside == 2 && k >= 1) WKV_CUDA(cudaStreamWaitEvent(ds, g.freed[b ^ 1], 0), "cudaStreamWaitEvent(other)");
+        if ((st = flag_range(la, lb, ds)) != WIND_OK) return st;
+      }
+      WKV_CUDA(cudaEventRecord(g.freed[b], ds), "cudaEventRecord(freed)");
     } else {
-      if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(g.side, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
-      if ((st = dma(la, lb, i0, mk, g.buf[b])) != WIND_OK) return st;
-      WKV_CUDA(cudaEventRecord(g.ready[b], g.side), "cudaEventRecord(ready)");
+      if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(g.side[0], g.freed[b], 0), "cudaStreamWaitEvent(freed)");
+      if ((st = dma(la, lb, i0, mk, g.buf[b], g.side[0])) != WIND_OK) return st;
+      WKV_CUDA(cudaEventRecord(g.ready[b], g.side[0]), "cudaEventRecord(ready)");
       WKV_CUDA(cudaStreamWaitEvent(s, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
       OpItem si{&shadow, g.iota, dev_bt + i0, mk};
       if ((st = run_op(&stage, &si, 1, la, lb, s, HeadRange(), k == K - 1 ? &t_exposed : &t_hidden)) != WIND_OK)
@@ -925,8 +937,9 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
       WKV_CUDA(cudaEventRecord(g.freed[b], s), "cudaEventRecord(freed)");
     }
   }
-  if (out)  // join: the side stream's last copy and flags (it runs its work in order)
-    WKV_CUDA(cudaStreamWaitEvent(s, g.freed[(K - 1) & 1], 0), "cudaStreamWaitEvent(join)");
+  if (out)  // join: each DMA stream's last copy and flags (each runs its work in order)
+    for (int q = 0; q < nside; ++q)
+      WKV_CUDA(cudaStreamWaitEvent(s, g.freed[(K - 1 - q) & 1], 0), "cudaStreamWaitEvent(join)");
   if (!capturing) {
     WKV_CUDA(cudaEventRecord(g.done, s), "cudaEventRecord(done)");
     g.has_done = true;
