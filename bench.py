@@ -613,6 +613,21 @@ def run_pressure(wk, device, reps: int = 3) -> dict:
     out["swap_out_plus_incoming_ms"] = round(t_both, 2)
     out["paper_claim"] = ("rescheduling (migration) instead of swapping frees the decode pool "
                           f"{t_swap / out['evict_by_migration_ms_cap16']:.0f}x faster at an NVLink-rate cap")
+    # full-duplex PCIe: swap the victims out to a second host pool while the first host
+    # pool's copy (the earlier victims) swaps back in, on two streams (DistServe-style swap
+    # traffic both ways at once, P:130 / P:341); aggregate = both directions' payload
+    host2 = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, nv, loc="host")
+    back_t = torch.as_tensor(np.arange(nv, dtype=np.int32), device=dev)
+
+    def exchange():
+        s_swap.wait_stream(s_mig)
+        wk.swap_out(dpool, vt, host2, ht_h, stream=s_swap)
+        wk.swap_in(host, ht_h, other, back_t, stream=s_mig)
+        s_mig.wait_stream(s_swap)
+    t_x = time_device(exchange, reps, 1, s_mig) / reps
+    out["swap_exchange"] = {"ms": round(t_x, 2), "aggregate_gbs": round(2 * vb / t_x / 1e6, 1),
+                            "note": "swap-out and swap-in of 12.7 GiB each at the same time (staged paths)"}
+    host2.destroy()
     del dpool, host, other, src_inc
     return out
 

@@ -18,7 +18,7 @@ out = {}
 for cfg, nsw in [(c, n) for c, n in (("C1", None), ("C3", 64), ("C4", 400), ("C5", 4096)) if c in CFGS]:
     case = migration_case(cfg)
     sh = case.shape
-    n = nsw or case.n
+    n = int(os.environ.get("STAGED_N", 0)) or nsw or case.n
     n = min(n, case.n)
     src = bench.make_pool(wk, sh, case.nb_src, 0, case.content_seed, case.src_tag)
     host = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, n, loc="host")
