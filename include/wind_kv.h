@@ -62,7 +62,7 @@ typedef enum { WIND_LOC_DEVICE = 0, WIND_LOC_HOST = 1 /* pinned, mapped, portabl
 
 /* Pool flags. */
 #define WIND_POOL_DEBUG 0x1u /* ops into/out of this pool also run a device table check */
-#define WIND_POOL_NO_STAGING 0x2u /* host pools: no copy-engine staging (saves 2 x max(32 MiB,
+#define WIND_POOL_NO_STAGING 0x2u /* host pools: no copy-engine staging (saves 3 x max(32 MiB,
                                      2 L C) of device memory; swaps use the SM kernels) */
 
 /* Pool descriptor.  Layout (reading R2): [L][2][NB][H][bs][d] elements of
@@ -73,7 +73,7 @@ typedef enum { WIND_LOC_DEVICE = 0, WIND_LOC_HOST = 1 /* pinned, mapped, portabl
  * Requirements: every extent >= 1, n_layers <= WIND_KV_MAX_LAYERS, elem_bytes in {1,2,4}
  * (fp8 / fp16|bf16 / fp32 payloads are raw bytes, never interpreted: reading R13),
  * C % 16 == 0.  For a host pool, `device` names the GPU whose copy engines serve it: pool
- * creation also allocates there the staging of the staged swap path (2 buffers of
+ * creation also allocates there the staging of the staged swap path (3 buffers of
  * max(32 MiB, 2 * n_layers * C) bytes, a side stream, events; best effort — without a GPU
  * `device` the pool simply has no staging and swaps use the SM kernels). */
 typedef struct {
@@ -180,8 +180,8 @@ wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind
  *     pinned host memory) and the host pool has staging on the executing GPU: a TMA kernel
  *     gathers (scatters) the device blocks through the device table into a contiguous
  *     device staging buffer at HBM rate, and the copy engines move each chunk over PCIe,
- *     one cudaMemcpy2DAsync per run of adjacent host slots, double-buffered on a side
- *     stream (fork / join with events: graph-capturable).  Chunks are layer-major and
+ *     one cudaMemcpy2DAsync per run of adjacent host slots, triple-buffered on side
+ *     streams (fork / join with events: graph-capturable).  Chunks are layer-major and
  *     dst's layer flags move as each layer's last chunk lands (layer_wait works as for
  *     migrate).  host_bt is READ ON THE CPU at enqueue (entries out of range: BLOCK_RANGE,
  *     nothing enqueued).  Staged ops on one host pool serialise on its buffers

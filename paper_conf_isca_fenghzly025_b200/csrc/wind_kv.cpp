@@ -97,6 +97,8 @@ struct DevCtx {
 };
 
 constexpr int kMaxDevices = 64;
+constexpr int kStageBufs = 3;  // staging buffers per host pool: a gather (scatter) may run
+                               // two chunks ahead of the PCIe copies
 DevCtx g_dev[kMaxDevices];
 
 wind_status dev_ctx(int dev, DevCtx** out) {
@@ -240,20 +242,20 @@ struct wind_kv_pool {
   void* ipc_flags_base = nullptr;
   uint8_t uuid[16] = {};           // physical GPU of the memory (device pools)
   std::atomic<uint32_t> enqueued{0};
-  // Host pools: the staged copy-engine path (kernel 4, staged_host_op).  Two device buffers
+  // Host pools: the staged copy-engine path (kernel 4, staged_host_op).  Three device buffers
   // on desc.device that SMs gather into / scatter from at HBM rate while the DMA engines
   // move the other buffer over PCIe, the side stream the DMA runs on, and the events of the
   // two-buffer pipeline.  Allocated at pool creation; dev < 0 if that failed.
   struct Staging {
     int dev = -1;
-    uint8_t* buf[2] = {nullptr, nullptr};
+    uint8_t* buf[kStageBufs] = {};
     size_t buf_bytes = 0;
+    int nbufs = 0;                    // buffers in use (kStageBufs; WIND_KV_STAGE_BUFS=2 for A/B)
     int32_t* iota = nullptr;          // 0, 1, ..., iota_n - 1: the staging side's block table
     int32_t iota_n = 0;
     uint32_t* dummy_flags = nullptr;  // layer flags of the internal gather / scatter ops
     cudaStream_t side[2] = {nullptr, nullptr};  // DMA streams (swap out uses both)
-    cudaEvent_t fork = nullptr, done = nullptr, ready[2] = {nullptr, nullptr},
-                freed[2] = {nullptr, nullptr};
+    cudaEvent_t fork = nullptr, done = nullptr, ready[kStageBufs] = {}, freed[kStageBufs] = {};
     bool has_done = false;            // `done` marks the end of the last uncaptured staged op
   } stg;
 };
@@ -287,7 +289,7 @@ constexpr int32_t kStagingMaxBlocks = 1 << 16;
 void staging_free(wind_kv_pool::Staging& g) {
   if (g.dev < 0) return;
   DeviceGuard dg(g.dev);
-  for (int b = 0; b < 2; ++b) {
+  for (int b = 0; b < kStageBufs; ++b) {
     if (g.buf[b]) cudaFree(g.buf[b]);
     if (g.ready[b]) cudaEventDestroy(g.ready[b]);
     if (g.freed[b]) cudaEventDestroy(g.freed[b]);
@@ -302,7 +304,7 @@ void staging_free(wind_kv_pool::Staging& g) {
   g = wind_kv_pool::Staging();
 }
 
-// Staging of a host pool on device `dev`: 2 buffers of max(32 MiB, 2 * L * C) bytes (so one
+// Staging of a host pool on device `dev`: 3 buffers of max(32 MiB, 2 * L * C) bytes (so one
 // block of every layer always fits), the identity table, dummy flags, a side stream and
 // the pipeline events.  Best effort: on failure the pool has no staging and the HOST path
 // uses the SM kernels (mapped pinned memory).
@@ -319,8 +321,11 @@ void staging_init(wind_kv_pool* p, int dev) {
   g.iota_n = static_cast<int32_t>(std::min<int64_t>(kStagingMaxBlocks, g.buf_bytes / (2 * p->chunk)));
   std::vector<int32_t> iota(g.iota_n);
   for (int32_t i = 0; i < g.iota_n; ++i) iota[i] = i;
-  bool ok = cudaMalloc(&g.buf[0], g.buf_bytes) == cudaSuccess &&
-            cudaMalloc(&g.buf[1], g.buf_bytes) == cudaSuccess &&
+  g.nbufs = kStageBufs;
+  if (const char* e = getenv("WIND_KV_STAGE_BUFS")) g.nbufs = std::max(2, std::min(kStageBufs, atoi(e)));
+  bool ok = true;
+  for (int b = 0; ok && b < g.nbufs; ++b) ok = cudaMalloc(&g.buf[b], g.buf_bytes) == cudaSuccess;
+  ok = ok &&
             cudaMalloc(&g.iota, sizeof(int32_t) * g.iota_n) == cudaSuccess &&
             cudaMemcpy(g.iota, iota.data(), sizeof(int32_t) * g.iota_n, cudaMemcpyHostToDevice) == cudaSuccess &&
             cudaMalloc(&g.dummy_flags, sizeof(uint32_t) * WIND_KV_MAX_LAYERS) == cudaSuccess &&
@@ -329,7 +334,7 @@ void staging_init(wind_kv_pool* p, int dev) {
             cudaStreamCreateWithFlags(&g.side[1], cudaStreamNonBlocking) == cudaSuccess &&
             cudaEventCreateWithFlags(&g.fork, cudaEventDisableTiming) == cudaSuccess &&
             cudaEventCreateWithFlags(&g.done, cudaEventDisableTiming) == cudaSuccess;
-  for (int b = 0; ok && b < 2; ++b)
+  for (int b = 0; ok && b < kStageBufs; ++b)
     ok = cudaEventCreateWithFlags(&g.ready[b], cudaEventDisableTiming) == cudaSuccess &&
          cudaEventCreateWithFlags(&g.freed[b], cudaEventDisableTiming) == cudaSuccess;
   if (!ok) staging_free(g);
@@ -792,7 +797,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
 //     host slots, rows = the chunk's K/V planes, on a side stream.
 // Chunks are layer-major (A5): a chunk is a range of whole layers for all n blocks
 // when they fit the buffer, else one layer for a range of blocks.  They alternate between
-// two buffers, so the gather of chunk k + 1 overlaps the PCIe copy of chunk k (fork / join
+// three buffers, so gathers run up to two chunks ahead of the PCIe copies (fork / join
 // with events: graph-capturable).  dst's layer flags are published as each layer's last
 // chunk lands (after its PCIe copy on the side stream for a swap out, after its scatter on
 // the op's stream for a swap in), so a consumer can start on layer 0 of a swap-in while
@@ -904,29 +909,30 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
   };
   for (int32_t k = 0; k < K; ++k) {
     const int32_t la = lo + (k / bchunks) * lpc, lb = std::min(hi, la + lpc);
-    const int32_t i0 = (k % bchunks) * m, mk = std::min(m, it.n - i0), b = k & 1;
+    const int32_t i0 = (k % bchunks) * m, mk = std::min(m, it.n - i0), b = k % g.nbufs;
     const bool layers_done = k % bchunks == bchunks - 1;  // last block chunk of [la, lb)
     stage.base = g.buf[b];
     stage.desc.first_layer = la;
     stage.desc.n_layers = lb - la;
     stage.bytes = static_cast<size_t>(2 * (lb - la) * spitch);
     if (out) {
-      if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(s, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
+      if (k >= g.nbufs) WKV_CUDA(cudaStreamWaitEvent(s, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
       OpItem gi{&stage, dev_bt + i0, g.iota, mk};
       if ((st = run_op(dev, &gi, 1, la, lb, s, HeadRange(), k == 0 ? &t_exposed : &t_hidden)) != WIND_OK)
         return st;
-      cudaStream_t ds = g.side[b % nside];
+      cudaStream_t ds = g.side[k % nside];
       WKV_CUDA(cudaEventRecord(g.ready[b], s), "cudaEventRecord(ready)");
       WKV_CUDA(cudaStreamWaitEvent(ds, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
       if ((st = dma(la, lb, i0, mk, g.buf[b], ds)) != WIND_OK) return st;
       if (layers_done) {
         // the layers' earlier chunks may have gone over the other DMA stream
-        if (nside == 2 && k >= 1) WKV_CUDA(cudaStreamWaitEvent(ds, g.freed[b ^ 1], 0), "cudaStreamWaitEvent(other)");
+        if (nside == 2 && k >= 1)
+          WKV_CUDA(cudaStreamWaitEvent(ds, g.freed[(k - 1) % g.nbufs], 0), "cudaStreamWaitEvent(other)");
         if ((st = flag_range(la, lb, ds)) != WIND_OK) return st;
       }
       WKV_CUDA(cudaEventRecord(g.freed[b], ds), "cudaEventRecord(freed)");
     } else {
-      if (k >= 2) WKV_CUDA(cudaStreamWaitEvent(g.side[0], g.freed[b], 0), "cudaStreamWaitEvent(freed)");
+      if (k >= g.nbufs) WKV_CUDA(cudaStreamWaitEvent(g.side[0], g.freed[b], 0), "cudaStreamWaitEvent(freed)");
       if ((st = dma(la, lb, i0, mk, g.buf[b], g.side[0])) != WIND_OK) return st;
       WKV_CUDA(cudaEventRecord(g.ready[b], g.side[0]), "cudaEventRecord(ready)");
       WKV_CUDA(cudaStreamWaitEvent(s, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
@@ -939,7 +945,7 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
   }
   if (out)  // join: each DMA stream's last copy and flags (each runs its work in order)
     for (int q = 0; q < nside; ++q)
-      WKV_CUDA(cudaStreamWaitEvent(s, g.freed[(K - 1 - q) & 1], 0), "cudaStreamWaitEvent(join)");
+      WKV_CUDA(cudaStreamWaitEvent(s, g.freed[(K - 1 - q) % g.nbufs], 0), "cudaStreamWaitEvent(join)");
   if (!capturing) {
     WKV_CUDA(cudaEventRecord(g.done, s), "cudaEventRecord(done)");
     g.has_done = true;
