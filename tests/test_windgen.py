@@ -70,3 +70,17 @@ def test_hash_shuffle_uniformish():
     d = W.hash_shuffle_dest(8000, 8, 5)
     cnt = np.bincount(d, minlength=8)
     assert cnt.min() > 850 and cnt.max() < 1150
+
+
+def test_seed_offset_zero_is_the_survey_seeds_and_nonzero_changes_the_case():
+    """bench --seed: offset 0 reproduces S§8(d)'s seeds exactly; another offset draws a new
+    case from the same distributions (same request count, different lengths / slots /
+    content seed)."""
+    from windgen import migration_case
+    a, b = migration_case("C2"), migration_case("C2", seed_offset=0)
+    assert np.array_equal(a.src_bt, b.src_bt) and np.array_equal(a.dst_bt, b.dst_bt)
+    assert a.content_seed == b.content_seed == 3002
+    c = migration_case("C2", seed_offset=5)
+    assert c.lengths.size == a.lengths.size and c.content_seed == 3007
+    assert not np.array_equal(c.lengths, a.lengths)
+    assert c.lengths.min() >= 256 and c.lengths.max() <= 2048
