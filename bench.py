@@ -1082,9 +1082,25 @@ def run_gpu(args) -> None:
     if role in ("solo", "decode"):
         dst = make_pool(wk, sh, case.nb_dst, local, case.content_seed, case.dst_tag)
     if world > 1:
-        handles = parallel.exchange_handles(dst.export() if role == "decode" else None)
-        if role == "push":
-            dst = wk.Pool.import_(handles[partner], local)
+        # pair setup (CUDA IPC export / import): every rank reports whether it succeeded, so
+        # a failure prints one explanatory line instead of a traceback and a hung barrier
+        err = None
+        try:
+            handles = parallel.exchange_handles(dst.export() if role == "decode" else None)
+            if role == "push":
+                dst = wk.Pool.import_(handles[partner], local)
+        except Exception as e:  # noqa: BLE001 — reported below, then the run ends
+            err = f"rank {rank}: {type(e).__name__}: {e}"[:300]
+        errs: list = [None] * world
+        dist.all_gather_object(errs, err)
+        errs = [x for x in errs if x]
+        if errs:
+            if rank == 0:
+                print(json.dumps({"metric": METRIC, "value": None, "unit": "GB/s", "n_gpus": world,
+                                  "error": "peer pool setup failed: " + " | ".join(errs)}), flush=True)
+            dist.barrier()
+            dist.destroy_process_group()
+            raise SystemExit(1)
     stream = torch.cuda.Stream(local)
     sbt = torch.as_tensor(case.src_bt, device=dev)
     dbt = torch.as_tensor(case.dst_bt, device=dev)
