@@ -794,12 +794,13 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
 //   device side (any table, device-resident): a TMA gather (swap out) / scatter (swap in)
 //     kernel between the device pool and a contiguous staging buffer at HBM rate;
 //   host side (table read on the CPU at enqueue): one cudaMemcpy2DAsync per run of adjacent
-//     host slots, rows = the chunk's K/V planes, on a side stream.
+//     host slots, rows = the chunk's K/V planes, on side streams (a swap-out alternates its
+//     chunks over two: two D2H copies in flight drive PCIe harder than one).
 // Chunks are layer-major (A5): a chunk is a range of whole layers for all n blocks
 // when they fit the buffer, else one layer for a range of blocks.  They alternate between
 // three buffers, so gathers run up to two chunks ahead of the PCIe copies (fork / join
 // with events: graph-capturable).  dst's layer flags are published as each layer's last
-// chunk lands (after its PCIe copy on the side stream for a swap out, after its scatter on
+// chunk lands (after its PCIe copy on a side stream for a swap out, after its scatter on
 // the op's stream for a swap in), so a consumer can start on layer 0 of a swap-in while
 // later layers are still in flight.
 wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo, int32_t hi,
