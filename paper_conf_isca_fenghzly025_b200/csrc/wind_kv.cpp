@@ -156,6 +156,15 @@ wind_kv_tuning g_tune[3] = {
 //    them ahead of PCIe (56-57 / 55 GB/s) with 4-6 % victim cost (1.5 MiB+: no faster).
 constexpr int64_t kHostToHostInFlight = 384 << 10;
 
+// WIND_KV_PDL=0 launches the copy kernels without programmatic dependent launch (A/B).
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("WIND_KV_PDL");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+
 // WIND_KV_BLOCKED_DEALING=0 turns the small-op contiguous dealing off (A/B measurements).
 bool blocked_dealing_enabled() {
   static const bool on = [] {
@@ -1140,7 +1149,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   p.blocked = (p.units_per_plane < grid && t.rate_mbps == 0 && blocked_dealing_enabled()) ? 1 : 0;
   // rate limit: each of the `grid` CTAs gets rate / grid; ns per payload byte per CTA
   p.ns_per_byte = t.rate_mbps > 0 ? static_cast<float>(grid * 1e3 / t.rate_mbps) : 0.f;
-  cudaError_t e = launch_copy(p, kernel, static_cast<int>(grid), s);
+  cudaError_t e = launch_copy(p, kernel, static_cast<int>(grid), s, pdl_enabled());
   if (e != cudaSuccess) return cuda_fail(e, "copy kernel launch");
   g_launches += 1;
   for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);

@@ -76,7 +76,9 @@ cudaError_t launch_flag_bump(const Params& p, cudaStream_t s);
 cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s);
 
 // Launchers (wind_kv_kernels.cu).  Return cudaGetLastError() after the launch.
-cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s);
+// pdl: launch with programmatic stream serialization (the kernel's prologue may overlap the
+// previous kernel on the stream; it waits for it before touching global memory).
+cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s, bool pdl);
 size_t tma_smem_bytes(int stages, int stage_bytes);
 cudaError_t prepare_kernels(int device, size_t max_tma_smem);
 

@@ -177,6 +177,15 @@ __device__ __forceinline__ void st_stream_ef(int4* p, const int4& v, uint64_t po
                : "memory");
 }
 
+// Programmatic dependent launch (PDL): a copy kernel launched right behind another one on
+// its stream may start its prologue (shared-memory carve-out, mbarrier init) on SMs the
+// previous grid has left, then waits here for that grid to complete and flush before it
+// touches any global memory — data, flags or counters.  No-op without the launch attribute.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_launch_dependents() {
+  asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
+}
+
 __device__ __forceinline__ uint64_t globaltimer_ns() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -409,6 +418,7 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
+  pdl_wait();  // everything below may see the previous grid's writes
   if (blockIdx.x == 0 && threadIdx.x == 33) publish_untouched_layers(p);  // an idle consumer lane
   if (p.abort_word && *reinterpret_cast<const volatile int32_t*>(p.abort_word)) {
     if (blockIdx.x == 0 && threadIdx.x == 0) publish_aborted(p);
@@ -433,6 +443,10 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
       if (u >= uend) {
         if (lane == 0) desc[st].nseg = -1;
         mbar_arrive(&full[st]);
+        // every load of this CTA is issued: the next op on the stream may launch once all
+        // CTAs got here (its CTAs then take SMs as ours exit and wait in pdl_wait) — never
+        // earlier, so a paced op does not park the next op's CTAs on idle SMs
+        pdl_launch_dependents();
         break;
       }
       int32_t plane;
@@ -527,6 +541,7 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
   const int tid = threadIdx.x;
   const bool ef = p.evict_first != 0;
   const uint64_t pol = ef ? evict_first_policy() : 0;
+  pdl_wait();
   if (blockIdx.x == 0 && tid == 32) publish_untouched_layers(p);  // not the decoding warp
   if (p.abort_word && *reinterpret_cast<const volatile int32_t*>(p.abort_word)) {
     if (blockIdx.x == 0 && tid == 0) publish_aborted(p);
@@ -544,6 +559,7 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
   }
   Pacer pacer;
   for (int64_t u = u0; u < uend; u += ustep) {
+    if (u + ustep >= uend) pdl_launch_dependents();  // this CTA's last unit (uniform)
     if (tid < 32) {
       int32_t plane;
       uint32_t bytes;
@@ -674,13 +690,23 @@ cudaError_t prepare_kernels(int device, size_t max_tma_smem) {
   return cudaSuccess;
 }
 
-cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s) {
+cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s, bool pdl) {
+  cudaLaunchConfig_t cfg = {};
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.gridDim = dim3(static_cast<unsigned>(grid));
+  cfg.stream = s;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl ? 1 : 0;
   if (kernel == kTma) {
-    tma_copy_kernel<<<grid, 64, tma_smem_bytes(p.stages, p.stage_bytes), s>>>(p);
-  } else {
-    simt_copy_kernel<<<grid, kSimtThreads, 0, s>>>(p);
+    cfg.blockDim = dim3(64);
+    cfg.dynamicSmemBytes = tma_smem_bytes(p.stages, p.stage_bytes);
+    return cudaLaunchKernelEx(&cfg, tma_copy_kernel, p);
   }
-  return cudaGetLastError();
+  cfg.blockDim = dim3(kSimtThreads);
+  cfg.dynamicSmemBytes = 0;
+  return cudaLaunchKernelEx(&cfg, simt_copy_kernel, p);
 }
 
 cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s) {
