@@ -30,6 +30,13 @@
  *     be queued on one stream, where ops run in order).
  *   - `cudaStream_t` parameters are passed as `void*` (0 = the legacy default stream) so
  *     the header needs no CUDA include.
+ *   - The copy kernels use programmatic dependent launch: each waits for the previous
+ *     kernel on its stream to complete before touching global memory, and signals
+ *     programmatic completion once all its loads are issued.  Ordinary launches after an
+ *     op are unaffected; a kernel YOU launch after an op with programmatic stream
+ *     serialization must call cudaGridDependencySynchronize() before reading the op's
+ *     destination (the standard PDL contract).  WIND_KV_PDL=0 in the environment turns it
+ *     off.
  */
 #ifndef WIND_KV_H
 #define WIND_KV_H
