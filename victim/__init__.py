@@ -2,8 +2,8 @@
   * paged decode attention over a wind_kv pool: the co-running "decode stream" of the
     interference measurement (S§8(d)); validated against torch attention in
     tests/test_gpu_victim.py;
-  * copy-engine comparators (cudaMemcpyAsync per chunk, cudaMemcpyBatchAsync) for the same
-    paged gather (S§7 step 4)."""
+  * a copy-engine comparator (one cudaMemcpyAsync per chunk) for the same paged gather
+    (S§7 step 4)."""
 from __future__ import annotations
 
 import ctypes as ct
@@ -55,7 +55,7 @@ def _ce():
         if not os.path.exists(CE_LIB):
             raise ImportError(f"{CE_LIB} missing: run __graft_entry__.build()")
         L = ct.CDLL(CE_LIB)
-        for name in ("ce_gather_loop", "ce_gather_batch"):
+        for name in ("ce_gather_loop",):
             f = getattr(L, name)
             f.argtypes = [ct.c_void_p, ct.c_int64, ct.c_void_p, ct.c_int64, ct.c_int64, ct.c_void_p,
                           ct.c_void_p, ct.c_int32, ct.c_int32, ct.c_void_p]
@@ -84,11 +84,13 @@ def decode_attention(q, k_plane_ptr: int, v_plane_ptr: int, bt, ctx, hkv: int, b
 
 def ce_gather(kind: str, src_plane0: int, s_stride: int, dst_plane0: int, d_stride: int, chunk: int,
               src_bt: np.ndarray, dst_bt: np.ndarray, planes: int, stream: int) -> None:
-    """Copy-engine gather: kind 'loop' (cudaMemcpyAsync per chunk) or 'batch'
-    (cudaMemcpyBatchAsync).  Tables are host int32 arrays."""
+    """Copy-engine gather: kind 'loop' (one cudaMemcpyAsync per chunk), the only kind.
+    Tables are host int32 arrays."""
+    if kind != "loop":
+        raise ValueError(f"unknown copy-engine comparator {kind!r}")
     s = np.ascontiguousarray(src_bt, np.int32)
     d = np.ascontiguousarray(dst_bt, np.int32)
-    f = _ce().ce_gather_loop if kind == "loop" else _ce().ce_gather_batch
+    f = _ce().ce_gather_loop
     rc = f(src_plane0, s_stride, dst_plane0, d_stride, chunk, s.ctypes.data, d.ctypes.data, s.size,
            planes, stream or None)
     if rc != 0:
