@@ -158,8 +158,12 @@ wind_status wind_kv_pool_import(const wind_kv_ipc_handle* handle, int32_t local_
  *   Executing device: src's device if src is a device pool (its own, or the device an
  *     imported src was mapped into), else dst's.  `stream` must belong to it
  *     (INVALID_ARG otherwise).  Cross-device ops push over NVLink peer stores (or pull
- *     when src is the remote one); host pools move over PCIe (staged copy engines or
- *     mapped memory: see wind_kv_swap_out).
+ *     when src is the remote one); host pools move over PCIe (mapped memory by default,
+ *     staged copy engines on request: see wind_kv_swap_out).
+ *   Argument errors, nothing enqueued, in this order: INVALID_ARG (NULL pool, n_blocks < 0,
+ *     NULL table with n_blocks > 0, stream of another device, imported pool mapped for
+ *     another device), then GEOMETRY, then LAYER_RANGE, then NO_PEER / UNSUPPORTED
+ *     (unreachable pools, host -> host).
  *   Layer flags (A5): every call with n_blocks > 0 and lo < hi takes one ticket on dst
  *     (see wind_kv_layer_ticket) and, as each layer's bytes become visible, adds 1 to
  *     dst's layer_done flag of that layer with release semantics: at GPU scope when src
@@ -182,20 +186,25 @@ wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind
 
 /* swap_out / swap_in (A6): migrate over all layers of the device pool with a HOST pool as
  * destination / source.  The host pool must cover the device pool's
- * layers.  Executes on the device pool's GPU.  Two mechanisms (HOST path, kernel auto):
- *   - staged (kernel 4), chosen when the HOST-side table (host_bt) is host-readable (e.g.
- *     pinned host memory) and the host pool has staging on the executing GPU: a TMA kernel
- *     gathers (scatters) the device blocks through the device table into a contiguous
- *     device staging buffer at HBM rate, and the copy engines move each chunk over PCIe,
- *     one cudaMemcpy2DAsync per run of adjacent host slots, triple-buffered on side
- *     streams (fork / join with events: graph-capturable).  Chunks are layer-major and
- *     dst's layer flags move as each layer's last chunk lands (layer_wait works as for
- *     migrate).  host_bt is READ ON THE CPU at enqueue (entries out of range: BLOCK_RANGE,
- *     nothing enqueued).  Staged ops on one host pool serialise on its buffers
+ * layers.  Executes on the device pool's GPU.  Two mechanisms:
+ *   - default (HOST path, kernel 0 / 1 / 2): SM / TMA stores to and loads from mapped pinned
+ *     memory over PCIe, tables borrowed and read when the op executes (the migrate
+ *     contract), per-layer flags as in migrate.  Grids are sized by the bytes they keep in
+ *     flight (wind_kv_tuning.max_ctas).
+ *   - staged (kernel 4, OPT-IN via wind_kv_set_tuning(WIND_PATH_HOST) or a per-op
+ *     wind_kv_migrate_ex override; UNSUPPORTED when it does not apply): the HOST-side table
+ *     (host_bt) must be host-readable (e.g. pinned host memory) and the host pool must have
+ *     staging on the executing GPU.  A TMA kernel gathers (scatters) the device blocks
+ *     through the device table into a contiguous device staging buffer at HBM rate, and the
+ *     copy engines move each chunk over PCIe, one cudaMemcpy2DAsync per run of adjacent host
+ *     slots, triple-buffered on side streams (fork / join with events).  Chunks are
+ *     layer-major and dst's layer flags move as each layer's last chunk lands.  CONTRACT
+ *     DIFFERENCE: host_bt is READ ON THE CPU AT ENQUEUE (entries out of range: BLOCK_RANGE,
+ *     nothing enqueued), so it must hold its final values when the call is made; inside a
+ *     CUDA graph capture its contents are baked into the graph (a replay moves the slots
+ *     the table held at capture).  Staged ops on one host pool serialise on its buffers
  *     automatically outside graph capture (inside a capture, order them yourself); they
  *     must be enqueued by one host thread at a time (the pool's events are reused).
- *   - otherwise SM / TMA stores to and loads from mapped pinned memory over PCIe, per-layer
- *     flags as in migrate.
  * A host pool's layer flags live in mapped host memory and are updated without PCIe
  * atomics, so ops INTO one host pool must not overlap in time (ops on one stream never
  * do); the host observes swap_out progress by reading the flags. */
@@ -246,6 +255,15 @@ typedef struct {
 wind_status wind_kv_migrate_batch(const wind_kv_pool* src, const wind_kv_migrate_item* items,
                                   int32_t n_items, int32_t layer_lo, int32_t layer_hi,
                                   void* stream);
+
+/* Route query (diagnostics, tests): the device an op from src to dst executes on, its
+ * tuning path (WIND_PATH_INTRA: both pools on one physical GPU; WIND_PATH_PEER: device pools
+ * on different GPUs, NVLink peer stores / loads; WIND_PATH_HOST: one side is a host pool)
+ * and whether its layer flags are published at system scope (1) or GPU scope (0).  Same
+ * reachability checks as an op (NO_PEER, UNSUPPORTED for host -> host); enables peer access
+ * like an op would.  Any out pointer may be NULL. */
+wind_status wind_kv_route(const wind_kv_pool* src, const wind_kv_pool* dst, int32_t* exec_device,
+                          int32_t* path, int32_t* sys_scope);
 
 /* ------------------------------------------------------------- layer flags (A5) */
 
@@ -305,9 +323,9 @@ wind_status wind_kv_check_device_error(const wind_kv_pool* pool);
  * of another stream that CUDA maps onto the same queue waits behind them: raise
  * CUDA_DEVICE_MAX_CONNECTIONS (e.g. 32) and keep few streams; the TMA / SIMT kernels pace
  * inside the kernel and never hold a queue),
- * 4 = staged copy engines (HOST path only: see wind_kv_swap_out; UNSUPPORTED when it does
- * not apply), 0 = auto (INTRA: TMA; PEER: SIMT; HOST: staged when it applies and
- * rate_mbps == 0, else TMA), 1 = TMA bulk staged copy, 2 = SIMT 16-B vector copy.
+ * 4 = staged copy engines (HOST path only, opt-in: see wind_kv_swap_out; UNSUPPORTED when
+ * it does not apply), 0 = auto (INTRA: TMA; PEER: SIMT; HOST: TMA on mapped pinned memory),
+ * 1 = TMA bulk staged copy, 2 = SIMT 16-B vector copy.
  * ctas_per_sm, stage_bytes (TMA stage / SIMT unit bytes, multiple of 16), stages (TMA ring
  * depth); 0 keeps the current value. */
 typedef enum { WIND_PATH_INTRA = 0, WIND_PATH_PEER = 1, WIND_PATH_HOST = 2 } wind_path;

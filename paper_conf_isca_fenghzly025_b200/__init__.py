@@ -20,7 +20,7 @@ import numpy as np
 
 __all__ = [
     "WindKVError", "Pool", "lib", "migrate", "migrate_batch", "migrate_heads", "swap_out", "swap_in", "compact",
-    "layer_wait", "validate", "plan_compact", "plan_rebalance", "check_device_error",
+    "layer_wait", "route", "validate", "plan_compact", "plan_rebalance", "check_device_error",
     "set_tuning", "get_tuning", "launch_count", "STATUS", "PATH_INTRA", "PATH_PEER", "PATH_HOST",
     "KERNEL_AUTO", "KERNEL_TMA", "KERNEL_SIMT", "EXPORTED_SYMBOLS", "Partition",
 ]
@@ -52,7 +52,7 @@ EXPORTED_SYMBOLS = [
     "wind_kv_plan_rebalance", "wind_kv_check_device_error", "wind_kv_set_tuning",
     "wind_kv_get_tuning", "wind_kv_migrate_ex", "wind_kv_launch_count", "wind_kv_status_string",
     "wind_kv_last_error",
-    "wind_kv_version", "wind_kv_partition_sms", "wind_kv_partition_destroy",
+    "wind_kv_version", "wind_kv_partition_sms", "wind_kv_partition_destroy", "wind_kv_route",
 ]
 
 
@@ -129,6 +129,7 @@ def lib() -> ct.CDLL:
         "wind_kv_migrate_ex": [P, P, P, P, I32, I32, I32, ct.POINTER(Tuning), P],
         "wind_kv_partition_sms": [I32, I32, ct.POINTER(SmPartition)],
         "wind_kv_partition_destroy": [ct.POINTER(SmPartition)],
+        "wind_kv_route": [P, P, ct.POINTER(I32), ct.POINTER(I32), ct.POINTER(I32)],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -162,10 +163,13 @@ def _ptr(x) -> Optional[int]:
         return x
     if hasattr(x, "data_ptr"):
         import torch
-        if x.dtype not in (torch.int32, torch.uint8):
-            raise TypeError("tables must be int32 tensors")
+        if x.dtype != torch.int32:
+            raise TypeError(f"block tables must be int32 tensors, got {x.dtype}")
         if not x.is_contiguous():
             raise ValueError("tables must be contiguous")
+        if not x.is_cuda and not x.is_pinned():
+            # the kernels read tables on the device: pageable host memory is not accessible
+            raise ValueError("block tables must be device tensors or pinned host tensors")
         return x.data_ptr()
     raise TypeError(f"cannot pass {type(x).__name__} as a device pointer")
 
@@ -379,6 +383,14 @@ def compact(pool: Pool, src_bt, dst_bt, n: Optional[int] = None, stream=None) ->
     n = _len(src_bt) if n is None else n
     _check(lib().wind_kv_compact(pool.handle, _ptr(src_bt), _ptr(dst_bt), n,
                                  _stream(stream, pool.device)))
+
+
+def route(src: Pool, dst: Pool) -> tuple[int, int, bool]:
+    """wind_kv_route: (executing device, path PATH_INTRA / PATH_PEER / PATH_HOST, system-scope
+    flag publication) of an op from src to dst."""
+    e, p, s = ct.c_int32(), ct.c_int32(), ct.c_int32()
+    _check(lib().wind_kv_route(src.handle, dst.handle, ct.byref(e), ct.byref(p), ct.byref(s)))
+    return int(e.value), int(p.value), bool(s.value)
 
 
 def layer_wait(dst: Pool, layer: int, ticket: int, stream=None) -> None:

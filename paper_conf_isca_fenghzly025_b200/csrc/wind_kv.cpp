@@ -137,8 +137,8 @@ wind_kv_tuning g_tune[3] = {
     // threads keep ~3 MiB of stores in flight (> 2 us x 900 GB/s) and leave SMs to the
     // co-running prefill / decode.  Not yet tuned on a multi-GPU box (one GPU per round-1 call).
     /* PEER  */ {kSimt, 1, 32768, 6, 96, 0, 0},
-    // HOST: PCIe-bound.  auto = the staged copy-engine path when the host table is
-    // host-readable (staged_host_op), else the TMA kernel on mapped pinned memory.
+    // HOST: PCIe-bound.  auto = the TMA kernel on mapped pinned memory (the staged copy-engine
+    // path, staged_host_op, is opt-in: kernel 4).
     // max_ctas 0 = per-direction defaults (kHostCtas*): SM stores to host memory beyond
     // what PCIe drains back up into the GPU's memory system — 8 TMA CTAs writing at 52 GB/s
     // slowed a co-running decode kernel by 73 %, 2 CTAs at the same rate by 2 %
@@ -621,30 +621,62 @@ struct HeadRange {
   int32_t src_lo = 0, dst_lo = 0, n = -1;
 };
 
-// Argument checks shared by every op: INVALID_ARG > GEOMETRY > LAYER_RANGE.
-wind_status check_args(const wind_kv_pool* src, const wind_kv_pool* dst, int32_t n, int32_t lo,
-                       int32_t hi, const HeadRange& hr = HeadRange()) {
+// Argument checks, split by precedence class (S§8(b) "Errors": INVALID_ARG, then GEOMETRY,
+// then LAYER_RANGE, then NO_PEER).  INVALID_ARG part of one (src, dst) pair: NULL pools,
+// n < 0, NULL tables of a non-empty op, bad head-range arguments.
+wind_status check_invalid(const wind_kv_pool* src, const wind_kv_pool* dst, int32_t n,
+                          const int32_t* sbt, const int32_t* dbt, const HeadRange& hr = HeadRange()) {
   if (!src || !dst) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
   if (n < 0) return fail(WIND_ERR_INVALID_ARG, "n_blocks < 0");
+  if (n > 0 && (!sbt || !dbt)) return fail(WIND_ERR_INVALID_ARG, "block table is NULL");
+  if (hr.n >= 0 && (hr.n < 1 || hr.src_lo < 0 || hr.dst_lo < 0))
+    return fail(WIND_ERR_INVALID_ARG, "head range: n_heads >= 1 and offsets >= 0 required");
+  return WIND_OK;
+}
+
+// GEOMETRY (and the head-tile UNSUPPORTED of a head range) of one pair.
+wind_status check_geometry(const wind_kv_pool* src, const wind_kv_pool* dst,
+                           const HeadRange& hr = HeadRange()) {
   if (hr.n < 0) {
     if (!same_geometry(src->desc, dst->desc))
       return fail(WIND_ERR_GEOMETRY, "pools differ in H/d/block_size/elem_bytes");
-  } else {
-    if (hr.n < 1 || hr.src_lo < 0 || hr.dst_lo < 0)
-      return fail(WIND_ERR_INVALID_ARG, "head range: n_heads >= 1 and offsets >= 0 required");
-    const wind_kv_pool_desc &a = src->desc, &b = dst->desc;
-    if (a.head_dim != b.head_dim || a.block_size != b.block_size || a.elem_bytes != b.elem_bytes)
-      return fail(WIND_ERR_GEOMETRY, "pools differ in d/block_size/elem_bytes");
-    if (hr.src_lo + hr.n > a.n_kv_heads || hr.dst_lo + hr.n > b.n_kv_heads)
-      return fail(WIND_ERR_GEOMETRY, "head range leaves a pool (src %d+%d of %d, dst %d+%d of %d)",
-                  hr.src_lo, hr.n, a.n_kv_heads, hr.dst_lo, hr.n, b.n_kv_heads);
-    if ((static_cast<int64_t>(a.block_size) * a.head_dim * a.elem_bytes) % 16 != 0)
-      return fail(WIND_ERR_UNSUPPORTED, "head tile bs*d*e_b must be a multiple of 16 bytes");
+    return WIND_OK;
   }
+  const wind_kv_pool_desc &a = src->desc, &b = dst->desc;
+  if (a.head_dim != b.head_dim || a.block_size != b.block_size || a.elem_bytes != b.elem_bytes)
+    return fail(WIND_ERR_GEOMETRY, "pools differ in d/block_size/elem_bytes");
+  if (hr.src_lo + hr.n > a.n_kv_heads || hr.dst_lo + hr.n > b.n_kv_heads)
+    return fail(WIND_ERR_GEOMETRY, "head range leaves a pool (src %d+%d of %d, dst %d+%d of %d)",
+                hr.src_lo, hr.n, a.n_kv_heads, hr.dst_lo, hr.n, b.n_kv_heads);
+  if ((static_cast<int64_t>(a.block_size) * a.head_dim * a.elem_bytes) % 16 != 0)
+    return fail(WIND_ERR_UNSUPPORTED, "head tile bs*d*e_b must be a multiple of 16 bytes");
+  return WIND_OK;
+}
+
+// LAYER_RANGE of one pair: lo <= hi, and a non-empty [lo, hi) inside both pools.
+wind_status check_layers(const wind_kv_pool* src, const wind_kv_pool* dst, int32_t lo, int32_t hi) {
   if (lo > hi) return fail(WIND_ERR_LAYER_RANGE, "layer_lo %d > layer_hi %d", lo, hi);
   if (lo < hi && (!layers_inside(src->desc, lo, hi) || !layers_inside(dst->desc, lo, hi)))
     return fail(WIND_ERR_LAYER_RANGE, "layers [%d, %d) not inside both pools", lo, hi);
   return WIND_OK;
+}
+
+// All argument checks of one pair in precedence order (wind_kv_validate; no stream).
+wind_status check_args(const wind_kv_pool* src, const wind_kv_pool* dst, int32_t n,
+                       const int32_t* sbt, const int32_t* dbt, int32_t lo, int32_t hi,
+                       const HeadRange& hr = HeadRange()) {
+  wind_status st;
+  if ((st = check_invalid(src, dst, n, sbt, dbt, hr)) != WIND_OK) return st;
+  if ((st = check_geometry(src, dst, hr)) != WIND_OK) return st;
+  return check_layers(src, dst, lo, hi);
+}
+
+// The device an op executes on (wind_kv.h, wind_kv_migrate): src's device if src is a
+// device pool, else dst's; -1 for host -> host (no executing device: UNSUPPORTED in route).
+int exec_device_of(const wind_kv_pool* src, const wind_kv_pool* dst) {
+  if (src->desc.loc == WIND_LOC_DEVICE) return src->desc.device;
+  if (dst->desc.loc == WIND_LOC_DEVICE) return dst->desc.device;
+  return -1;
 }
 
 // Which device runs the op, and which tuning path applies.
@@ -660,11 +692,6 @@ wind_status route(const wind_kv_pool* src, const wind_kv_pool* dst, int* exec, i
   *path = same_gpu ? WIND_PATH_INTRA : WIND_PATH_PEER;
   if (src->imported && dst->imported)
     return fail(WIND_ERR_UNSUPPORTED, "at least one pool must be local to this process");
-  // an imported pool is mapped for the device it was imported into: the op must run there
-  const wind_kv_pool* imp = src->imported ? src : (dst->imported ? dst : nullptr);
-  if (imp && imp->desc.device != *exec)
-    return fail(WIND_ERR_INVALID_ARG, "imported pool is mapped for device %d but the op executes on %d",
-                imp->desc.device, *exec);
   // a local pool on another device of this process: enable peer access from the executing one
   const wind_kv_pool* other = (src->desc.device != *exec) ? src : dst;
   if (!other->imported && other->desc.device != *exec) {
@@ -741,8 +768,8 @@ bool host_readable(const void* ptr) {
 // each pool's plane stride).  The tables must be host-readable (the driver needs every
 // address at enqueue time); the layer flags are published by one tiny kernel afterwards
 // (stream order: after every copy), so per-layer streaming is not available on this path.
-wind_status copy_engine_op(const Params& p, const OpItem* items, int n_items, cudaStream_t s,
-                           int32_t rate_mbps) {
+wind_status copy_engine_op(const Params& p, int32_t src_nb, const OpItem* items, int n_items,
+                           cudaStream_t s, int32_t rate_mbps) {
   const size_t rows = static_cast<size_t>(2) * p.n_layers;
   // rate limit: a pace kernel stamps the op start; after copies worth >= 20 us of the
   // budget, a pace kernel holds the stream until start + bytes_so_far / rate.  The stamp
@@ -750,6 +777,19 @@ wind_status copy_engine_op(const Params& p, const OpItem* items, int n_items, cu
   unsigned long long* t0 = reinterpret_cast<unsigned long long*>(p.counters + WIND_KV_MAX_LAYERS - 2);
   double sched_ns = 0, last_paced = 0;
   int launches = 0;
+  // the tables are read here, on the CPU: check them before anything is enqueued (an entry
+  // out of range would make a DMA copy write outside both pools)
+  for (int j = 0; j < n_items; ++j) {
+    const OpItem& it = items[j];
+    if (it.n == 0) continue;
+    if (!host_readable(it.sbt) || !host_readable(it.dbt))
+      return fail(WIND_ERR_UNSUPPORTED, "copy-engine path needs host-readable block tables");
+    for (int32_t i = 0; i < it.n; ++i)
+      if (static_cast<uint32_t>(it.sbt[i]) >= static_cast<uint32_t>(src_nb) ||
+          static_cast<uint32_t>(it.dbt[i]) >= static_cast<uint32_t>(it.dst->desc.n_blocks))
+        return fail(WIND_ERR_BLOCK_RANGE, "item %d: table entry %d out of range (src %d of %d, dst %d of %d)",
+                    j, i, it.sbt[i], src_nb, it.dbt[i], it.dst->desc.n_blocks);
+  }
   if (rate_mbps > 0) {
     WKV_CUDA(launch_pace(t0, 0, 1, s), "pace kernel launch");
     ++launches;
@@ -757,8 +797,6 @@ wind_status copy_engine_op(const Params& p, const OpItem* items, int n_items, cu
   for (int j = 0; j < n_items; ++j) {
     const OpItem& it = items[j];
     if (it.n == 0) continue;
-    if (!host_readable(it.sbt) || !host_readable(it.dbt))
-      return fail(WIND_ERR_UNSUPPORTED, "copy-engine path needs host-readable block tables");
     const Item& q = p.items[j];
     const bool co = q.coalesce != 0;
     for (int32_t i = 0; i < it.n;) {
@@ -793,8 +831,8 @@ wind_status copy_engine_op(const Params& p, const OpItem* items, int n_items, cu
 wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
                    int32_t hi, void* stream, const HeadRange& hr, const wind_kv_tuning* override_tuning);
 
-// Staged copy-engine host path (kernel 4; the HOST path's automatic choice when the
-// host-side block table is host-readable).  PCIe is the bottleneck of a swap, and the DMA
+// Staged copy-engine host path (kernel 4, opt-in: the host-side block table is read on the
+// CPU at enqueue, unlike every other op's tables).  PCIe is the bottleneck of a swap, and the DMA
 // engines drive it harder than SM stores to mapped memory (full-size write packets: 57 vs
 // 52 GB/s D2H on B200, profiles/r01/host_sweep.txt) while holding no SM; but a DMA engine
 // needs every address at enqueue time and pays a setup per copy, so it cannot follow a
@@ -979,20 +1017,35 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   } nvtx_range;
   int exec = -1, path = 0;
   wind_status st;
+  // (1) INVALID_ARG, every item: NULL pools / tables, n < 0, head-range arguments, repeated
+  // batch destinations, items on different executing devices, an imported pool mapped for
+  // another device, the stream's device (S§8(b) "Errors" precedence)
   for (int j = 0; j < n_items; ++j) {
-    if ((st = check_args(src, items[j].dst, items[j].n, lo, hi, hr)) != WIND_OK) return st;
-    if (items[j].n > 0 && (!items[j].sbt || !items[j].dbt)) return fail(WIND_ERR_INVALID_ARG, "block table is NULL");
+    const OpItem& it = items[j];
+    if ((st = check_invalid(src, it.dst, it.n, it.sbt, it.dbt, hr)) != WIND_OK) return st;
     for (int k = 0; k < j; ++k)
-      if (items[k].dst == items[j].dst) return fail(WIND_ERR_INVALID_ARG, "batch destinations must be distinct");
+      if (items[k].dst == it.dst) return fail(WIND_ERR_INVALID_ARG, "batch destinations must be distinct");
+    const int e2 = exec_device_of(src, it.dst);
+    if (j == 0) exec = e2;
+    else if (e2 != exec) return fail(WIND_ERR_INVALID_ARG, "batch items execute on different devices");
+    // an imported pool is mapped for the device it was imported into: the op must run there
+    const wind_kv_pool* imp = src->imported ? src : (it.dst->imported ? it.dst : nullptr);
+    if (imp && exec >= 0 && imp->desc.device != exec)
+      return fail(WIND_ERR_INVALID_ARG, "imported pool is mapped for device %d but the op executes on %d",
+                  imp->desc.device, exec);
   }
+  if (exec >= 0 && (st = check_stream(stream, exec)) != WIND_OK) return st;
+  // (2) GEOMETRY, then (3) LAYER_RANGE, over every item
+  for (int j = 0; j < n_items; ++j)
+    if ((st = check_geometry(src, items[j].dst, hr)) != WIND_OK) return st;
+  for (int j = 0; j < n_items; ++j)
+    if ((st = check_layers(src, items[j].dst, lo, hi)) != WIND_OK) return st;
+  // (4) reachability: NO_PEER (enables peer access as a side effect), UNSUPPORTED pairings
   for (int j = 0; j < n_items; ++j) {
     int e2 = -1, p2 = 0;
     if ((st = route(src, items[j].dst, &e2, &p2)) != WIND_OK) return st;
-    if (j == 0) { exec = e2; path = p2; }
-    else if (e2 != exec) return fail(WIND_ERR_INVALID_ARG, "batch items execute on different devices");
-    else path = std::max(path, p2);
+    path = j == 0 ? p2 : std::max(path, p2);
   }
-  if ((st = check_stream(stream, exec)) != WIND_OK) return st;
   int64_t total_n = 0;
   for (int j = 0; j < n_items; ++j) total_n += items[j].n;
   if (lo == hi || total_n == 0) return WIND_OK;  // R19: successful no-op, no ticket
@@ -1016,21 +1069,22 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
       debug = true;
     }
 
-  // HOST path, auto: the staged copy-engine path when it applies (one item, whole chunks,
-  // no rate limit, no debug pool, the host pool has staging on this device and its table is
-  // host-readable), else the TMA kernel over mapped pinned memory.
-  if (path == WIND_PATH_HOST && (t.kernel == kStaged || (t.kernel == kAuto && t.rate_mbps == 0))) {
+  // HOST path: the staged copy-engine path only when the caller asks for it (kernel 4, via
+  // wind_kv_set_tuning or a per-op wind_kv_migrate_ex override).  It reads the host-side
+  // table on the CPU at enqueue, which is a different contract from every other op's
+  // (tables borrowed and read when the op executes), so it is never chosen automatically:
+  // kernel 0 on the HOST path is the TMA kernel over mapped pinned memory.
+  if (path == WIND_PATH_HOST && t.kernel == kStaged) {
     const wind_kv_pool* host = src->desc.loc == WIND_LOC_HOST ? src : items[0].dst;
     const int32_t* hbt = host == src ? items[0].sbt : items[0].dbt;
     const bool staged = n_items == 1 && hr.n < 0 && !debug && host->stg.dev == exec &&
                         t.rate_mbps == 0 && host_readable(hbt);
-    if (staged)  // hidden chunks run the staged kernel tuning (4 x 48 KiB stages)
-      return staged_host_op(src, items[0], lo, hi, s,
-                            t.max_ctas > 0 ? t.max_ctas
-                                           : staged_hidden_ctas(src->chunk));
-    if (t.kernel == kStaged)
+    if (!staged)
       return fail(WIND_ERR_UNSUPPORTED, "staged path needs one item, whole chunks, no rate limit, a "
                   "host-readable host table and host-pool staging on device %d", exec);
+    // hidden chunks run the staged kernel tuning (4 x 48 KiB stages)
+    return staged_host_op(src, items[0], lo, hi, s,
+                          t.max_ctas > 0 ? t.max_ctas : staged_hidden_ctas(src->chunk));
   }
   const int kernel = t.kernel == kAuto ? (path == WIND_PATH_PEER ? kSimt : kTma) : t.kernel;
   if (kernel == kStaged)
@@ -1121,7 +1175,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     p.total_units = static_cast<int64_t>(2) * p.n_layers * p.units_per_plane;
   }
   if (kernel == kCopyEngine) {
-    if ((st = copy_engine_op(p, items, n_items, s, t.rate_mbps)) != WIND_OK) return st;
+    if ((st = copy_engine_op(p, src->desc.n_blocks, items, n_items, s, t.rate_mbps)) != WIND_OK) return st;
     for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
     return WIND_OK;
   }
@@ -1221,6 +1275,24 @@ extern "C" wind_status wind_kv_compact(wind_kv_pool* pool, const int32_t* src_bt
                          pool->desc.first_layer + pool->desc.n_layers, stream);
 }
 
+// Which device and path an op from src to dst takes (tests and diagnostics: a green
+// multi-device test must have run the PEER route, not INTRA).
+extern "C" wind_status wind_kv_route(const wind_kv_pool* src, const wind_kv_pool* dst,
+                                     int32_t* exec_device, int32_t* path, int32_t* sys_scope) {
+  if (!src || !dst) return fail(WIND_ERR_INVALID_ARG, "pool is NULL");
+  int exec = -1, pth = 0;
+  wind_status st = route(src, dst, &exec, &pth);
+  if (st != WIND_OK) return st;
+  if (exec_device) *exec_device = exec;
+  if (path) *path = pth;
+  // the publication scope run_op chooses: GPU scope only when both pools are device pools on
+  // the executing GPU
+  if (sys_scope)
+    *sys_scope = !(src->desc.loc == WIND_LOC_DEVICE && dst->desc.loc == WIND_LOC_DEVICE &&
+                   memcmp(src->uuid, dst->uuid, 16) == 0);
+  return WIND_OK;
+}
+
 // ------------------------------------------------------------------- layer flags
 
 extern "C" wind_status wind_kv_layer_ticket(const wind_kv_pool* dst, uint32_t* ticket) {
@@ -1275,9 +1347,8 @@ extern "C" wind_status wind_kv_layer_count(const wind_kv_pool* dst, int32_t laye
 extern "C" wind_status wind_kv_validate(const wind_kv_pool* src, const int32_t* sbt,
                                         const wind_kv_pool* dst, const int32_t* dbt, int32_t n,
                                         int32_t lo, int32_t hi) {
-  wind_status st = check_args(src, dst, n, lo, hi);
+  wind_status st = check_args(src, dst, n, sbt, dbt, lo, hi);
   if (st != WIND_OK) return st;
-  if (n > 0 && (!sbt || !dbt)) return fail(WIND_ERR_INVALID_ARG, "block table is NULL");
   return check_tables_host(src, sbt, dst, dbt, n);
 }
 

@@ -119,3 +119,19 @@ def test_null_arguments_fail_cleanly_without_gpu():
     assert L.wind_kv_pool_create(None, None, None) == -1
     assert L.wind_kv_pool_destroy(None) == 0
     assert "NULL" in wk.last_error()
+    assert L.wind_kv_route(None, None, None, None, None) == -1
+
+
+def test_binding_accepts_only_int32_device_accessible_tables():
+    """The binding marshals block tables as raw int32 addresses the kernels read on the
+    device: other dtypes would be reinterpreted, pageable host memory is not accessible."""
+    import torch
+    with pytest.raises(TypeError):
+        wk._ptr(torch.zeros(4, dtype=torch.uint8))
+    with pytest.raises(TypeError):
+        wk._ptr(torch.zeros(4, dtype=torch.int64))
+    with pytest.raises(ValueError):
+        wk._ptr(torch.zeros(4, dtype=torch.int32))  # pageable CPU memory
+    with pytest.raises(ValueError):
+        wk._ptr(torch.zeros(8, dtype=torch.int32)[::2])  # not contiguous
+    assert wk._ptr(None) is None and wk._ptr(1234) == 1234

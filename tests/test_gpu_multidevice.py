@@ -3,10 +3,12 @@ devices of one process — push (A4, prefill -> decode hand-off, executes on the
 GPU), pull, one-launch all-to-all to several devices (A8), host swaps served by another
 GPU's copy engines — and the multi-process CUDA IPC push across devices.
 
-The tests use device 1 (and up to 4 devices) when the box has them; on a one-GPU box every
-"peer" is device 0, which runs the same code through the intra-device route — the test
-logic is exercised either way, the NVLink route only on a multi-GPU box.  Every result is
-compared byte for byte with the CPU oracle over the whole destination pool.
+Cross-device tests need as many GPUs as they name and are SKIPPED otherwise (a one-GPU
+box would only run the intra-device route and prove nothing about NVLink); when they run
+they assert, through wind_kv_route, that the op took the PEER route with system-scope flag
+publication.  The one-launch all-to-all also runs with every pool on device 0, asserting
+the INTRA route, so its batching logic is covered on any box.  Every result is compared
+byte for byte with the CPU oracle over the whole destination pool.
 """
 import multiprocessing as mp
 import os
@@ -26,8 +28,18 @@ SHAPE_ARGS = (SH.n_layers, SH.n_kv_heads, SH.head_dim, SH.block_size, SH.elem_by
 
 
 def devices(k: int) -> list:
+    """k distinct GPUs, or skip: a cross-device test on fewer GPUs would silently run the
+    intra-device route instead of the one it names."""
     n = torch.cuda.device_count()
-    return [i % n for i in range(k)]
+    if n < k:
+        pytest.skip(f"needs {k} GPUs (NVLink peer route), this box has {n}")
+    return list(range(k))
+
+
+def assert_route(src: wk.Pool, dst: wk.Pool, exec_dev: int, path: int) -> None:
+    e, p, sys_scope = wk.route(src, dst)
+    assert (e, p) == (exec_dev, path), (e, p)
+    assert sys_scope == (path != wk.PATH_INTRA)
 
 
 def geom(p: wk.Pool) -> O.Geom:
@@ -79,6 +91,7 @@ def test_push_then_pull_across_devices():
     sbt = rng.permutation(150)[:77].astype(np.int32)
     dbt = rng.permutation(120)[:77].astype(np.int32)
     sa, sb = torch.cuda.Stream(device=a), torch.cuda.Stream(device=b)
+    assert_route(src, dst, a, wk.PATH_PEER)
     wk.migrate(src, tab(sbt, a), dst, tab(dbt, a), layer_lo=1, layer_hi=4, stream=sa)
     t = dst.layer_ticket()
     for l in range(4):
@@ -92,17 +105,21 @@ def test_push_then_pull_across_devices():
     np.testing.assert_array_equal(read(dst), want)
     back, k0 = pool(40, 3, a)
     pbt = np.arange(5, 35, dtype=np.int32)
+    assert_route(dst, back, b, wk.PATH_PEER)
     wk.migrate(dst, tab(dbt[:30], b), back, tab(pbt, b), stream=sb)
     want_b = k0.copy()
     assert O.migrate(want, geom(dst), dbt[:30], want_b, geom(back), pbt, 0, 4) == O.OK
     np.testing.assert_array_equal(read(back), want_b)
 
 
-def test_all_to_all_one_launch_per_device():
-    """A8 from one process: every device's pool pushes its outgoing blocks to every other
-    device's pool in ONE wind_kv_migrate_batch launch; destination slots are disjoint (the
-    planner's contract); every pool is byte-exact afterwards."""
-    devs = devices(4)
+@pytest.mark.parametrize("placement", ["peer", "same_device"])
+def test_all_to_all_one_launch_per_device(placement):
+    """A8 from one process: every pool pushes its outgoing blocks to every other pool in ONE
+    wind_kv_migrate_batch launch; destination slots are disjoint (the planner's contract);
+    every pool is byte-exact afterwards.  "peer": one pool on each of 2-4 GPUs (PEER route,
+    skipped on a one-GPU box); "same_device": 4 pools on device 0 (INTRA route)."""
+    devs = devices(2) + list(range(2, min(4, torch.cuda.device_count()))) if placement == "peer" \
+        else [0] * 4
     G, nb, per = len(devs), 200, 30
     pools = [pool(nb, 10 + g, devs[g]) for g in range(G)]
     before = [h.copy() for _, h in pools]
@@ -124,6 +141,9 @@ def test_all_to_all_one_launch_per_device():
             items.append((d, sb_, db_))
         plans.append(items)
     for s in range(G):
+        for d, _, _ in plans[s]:
+            assert_route(pools[s][0], pools[d][0], devs[s],
+                         wk.PATH_PEER if placement == "peer" else wk.PATH_INTRA)
         wk.migrate_batch(pools[s][0], [(pools[d][0], tab(sb_, devs[s]), tab(db_, devs[s]))
                                        for d, sb_, db_ in plans[s]], 0, SH.n_layers, stream=streams[s])
     for s in range(G):
@@ -139,8 +159,9 @@ def test_all_to_all_one_launch_per_device():
 @pytest.mark.parametrize("staging_device", ["same", "other"])
 def test_swap_from_second_device(staging_device):
     """A device pool on GPU b swaps out to / in from a host pool.  A host pool whose staging
-    lives on b takes the staged copy-engine path; one whose staging lives on another GPU
-    takes the SM path over mapped memory (the auto choice).  Both byte-exact."""
+    lives on b can take the opt-in staged copy-engine path; one whose staging lives on another
+    GPU only the SM path over mapped memory (the auto choice, which every case here uses).
+    Both byte-exact; the op executes on b."""
     a, b = devices(2)
     rng = np.random.default_rng(6)
     dev, d0 = pool(90, 20, b)
@@ -148,11 +169,11 @@ def test_swap_from_second_device(staging_device):
     hpin = torch.as_tensor(rng.permutation(70)[:60].astype(np.int32)).pin_memory()
     dbt = rng.permutation(90)[:60].astype(np.int32)
     sb = torch.cuda.Stream(device=b)
+    assert_route(dev, host, b, wk.PATH_HOST)
     n0 = wk.launch_count()
     wk.swap_out(dev, tab(dbt, b), host, hpin, stream=sb)
     sb.synchronize()
-    if staging_device == "other" and a != b:
-        assert wk.launch_count() - n0 == 1  # one SM kernel over mapped memory
+    assert wk.launch_count() - n0 == 1  # one SM kernel over mapped memory
     want_h = h0.copy()
     assert O.swap_out(d0, geom(dev), dbt, want_h, geom(host), hpin.numpy()) == O.OK
     np.testing.assert_array_equal(host.tensor().numpy(), want_h)
@@ -192,6 +213,7 @@ def test_ipc_push_across_devices():
     try:
         remote = wk.Pool.import_(q_out.get(timeout=300), a)
         src, s0 = pool(130, 30, a)
+        assert_route(src, remote, a, wk.PATH_PEER)
         rng = np.random.default_rng(7)
         sbt = rng.permutation(130)[:64].astype(np.int32)
         dbt = rng.permutation(100)[:64].astype(np.int32)

@@ -236,6 +236,50 @@ def test_argument_errors_match_oracle_precedence():
     torch.cuda.synchronize()
 
 
+def test_invalid_arg_precedes_geometry_and_layer_range():
+    """S§8(b) "Errors": every INVALID_ARG condition (NULL table, n < 0, repeated batch
+    destination, stream of another device) wins over GEOMETRY / LAYER_RANGE, with nothing
+    enqueued."""
+    sh = KVShape("t", 4, 2, 64, 2)
+    a, _ = make_pool(sh, 8, 1)
+    b, _ = make_pool(sh, 8, 2, first_layer=2)
+    c = wk.Pool(4, 4, 64, 16, 2, 8)  # different H: GEOMETRY against a
+    t1 = tab([1])
+    n0 = wk.launch_count()
+    # NULL table + geometry mismatch, NULL table + bad layer range
+    assert status_of(wk.migrate, a, None, c, t1, n=1, layer_lo=0, layer_hi=4) == -1
+    assert status_of(wk.migrate, a, t1, b, None, n=1, layer_lo=0, layer_hi=9) == -1
+    assert status_of(wk.migrate, a, None, b, t1, n=1, layer_lo=3, layer_hi=1) == -1
+    # n < 0 + geometry mismatch
+    assert status_of(wk.migrate, a, t1, c, t1, n=-1) == -1
+    # head range: n_heads < 1 beats a head range that leaves the pool
+    assert status_of(wk.migrate_heads, a, t1, c, t1, 0, 7, 0) == -1
+    # batch: a repeated destination beats another item's geometry mismatch
+    assert status_of(wk.migrate_batch, a, [(b, t1, t1), (c, t1, t1), (b, t1, t1)], 2, 4) == -1
+    # the same calls without the INVALID_ARG condition report the next class
+    assert status_of(wk.migrate, a, t1, c, t1, n=1, layer_lo=0, layer_hi=4) == -2
+    assert status_of(wk.migrate, a, t1, b, t1, n=1, layer_lo=0, layer_hi=9) == -3
+    assert status_of(wk.migrate_batch, a, [(b, t1, t1), (c, t1, t1)], 2, 4) == -2
+    assert wk.launch_count() == n0
+    assert a.layer_ticket() == b.layer_ticket() == c.layer_ticket() == 0
+    torch.cuda.synchronize()
+
+
+def test_wrong_device_stream_precedes_geometry():
+    """A stream of another device is INVALID_ARG even when the pools also mismatch (needs
+    two GPUs to build such a stream)."""
+    if torch.cuda.device_count() < 2:
+        pytest.skip("needs 2 GPUs for a stream of another device")
+    sh = KVShape("t", 4, 2, 64, 2)
+    a, _ = make_pool(sh, 8, 1)
+    c = wk.Pool(4, 4, 64, 16, 2, 8)
+    t1 = tab([1])
+    other = torch.cuda.Stream(device=1)
+    assert status_of(wk.migrate, a, t1, c, t1, n=1, stream=other) == -1
+    assert status_of(wk.migrate, a, t1, c, t1, n=1) == -2
+    assert status_of(wk.migrate, a, t1, a, tab([2]), n=1, layer_lo=0, layer_hi=9, stream=other) == -1
+
+
 def test_validate_matches_oracle_random_tables():
     sh = KVShape("t", 2, 2, 64, 2)
     a, _ = make_pool(sh, 6, 1)

@@ -1,7 +1,7 @@
-"""GPU parity of the staged copy-engine host path (A6 swap, kernel 4 / the HOST path's auto
-choice; wind_kv.h wind_kv_swap_out): a TMA gather / scatter between the device pool and a
-device staging buffer, the copy engines over PCIe per run of adjacent host slots, two
-buffers pipelined on a side stream.  Every result is compared with the CPU oracle over
+"""GPU parity of the staged copy-engine host path (A6 swap, kernel 4 — opt-in, selected
+here for every test by the autouse fixture; wind_kv.h wind_kv_swap_out): a TMA gather /
+scatter between the device pool and a device staging buffer, the copy engines over PCIe per
+run of adjacent host slots, buffers pipelined on side streams.  Every result is compared with the CPU oracle over
 the WHOLE host pool and device pool (untouched slots included), plus the layer flags.
 
 Chunking (layer-major): the staging buffer holds max(32 MiB, 2 L C) bytes; a chunk is as
@@ -25,6 +25,7 @@ DEV = torch.device("cuda", 0)
 @pytest.fixture(autouse=True)
 def default_tuning():
     saved = {p: wk.get_tuning(p) for p in (wk.PATH_INTRA, wk.PATH_PEER, wk.PATH_HOST)}
+    wk.set_tuning(wk.PATH_HOST, kernel=wk.KERNEL_STAGED)  # the staged path is opt-in
     yield
     for p, t in saved.items():
         wk.set_tuning(p, **t)
@@ -53,7 +54,7 @@ def dtab(a) -> torch.Tensor:
     return torch.as_tensor(np.asarray(a, np.int32), device=DEV)
 
 
-def htab(a) -> torch.Tensor:  # host-readable (pinned): selects the staged path
+def htab(a) -> torch.Tensor:  # host-readable (pinned): what the staged path needs
     return torch.as_tensor(np.asarray(a, np.int32)).pin_memory()
 
 
@@ -277,17 +278,47 @@ def test_staged_errors():
         wk.migrate_ex(dev, dtab(case.src_bt), other, dtab(case.src_bt),
                       wk.tuning(kernel=wk.KERNEL_STAGED))
     assert e.value.status == -10
-    # the auto choice falls back to the SM kernel for a device-resident host table
+    # the auto choice is the SM kernel over mapped memory, whatever the host table is
     wk.set_tuning(wk.PATH_HOST, kernel=wk.KERNEL_AUTO)
-    l0 = wk.launch_count()
-    wk.swap_out(dev, dtab(case.src_bt), host, dtab(np.arange(case.n)))
+    for ht in (dtab(np.arange(case.n)), htab(np.arange(case.n))):
+        l0 = wk.launch_count()
+        wk.swap_out(dev, dtab(case.src_bt), host, ht)
+        torch.cuda.synchronize()
+        assert wk.launch_count() - l0 == 1
+
+
+def test_default_host_path_reads_tables_when_it_executes():
+    """The default (auto) HOST path honours the borrowing contract: the tables are read when
+    the op executes on the stream, not at enqueue.  The stream is held by a sleep kernel, the
+    pinned host table is rewritten on the CPU after the swap_out was enqueued, and the
+    result must follow the REWRITTEN table (the staged path, which reads it at enqueue,
+    is opt-in for exactly this reason)."""
+    wk.set_tuning(wk.PATH_HOST, kernel=wk.KERNEL_AUTO)
+    case = migration_case("C1", scale=0.25)
+    sh = case.shape
+    n = case.n
+    dev, d0 = pool(sh, case.nb_src, 23)
+    host, h0 = pool(sh, n + 8, 24, loc="host")
+    first = np.arange(n, dtype=np.int32)
+    final = np.random.default_rng(25).permutation(n + 8)[:n].astype(np.int32)
+    ht = htab(first)
+    st = dtab(case.src_bt)
+    s = torch.cuda.Stream(DEV)
     torch.cuda.synchronize()
-    assert wk.launch_count() - l0 == 1
+    with torch.cuda.stream(s):
+        torch.cuda._sleep(200_000_000)  # ~0.1 s of device time before the swap runs
+    wk.swap_out(dev, st, host, ht, stream=s)
+    ht.copy_(torch.from_numpy(final))   # still before execution: the op must see this
+    s.synchronize()
+    want = h0.copy()
+    assert O.swap_out(d0, geom(dev), case.src_bt, want, geom(host), final) == O.OK
+    np.testing.assert_array_equal(host.tensor().numpy(), want)
 
 
 def test_no_staging_flag_uses_the_sm_path():
-    """WIND_POOL_NO_STAGING: the host pool gets no device staging, so even a host-readable
-    table takes the SM kernel over mapped memory (one launch); byte-exact either way."""
+    """WIND_POOL_NO_STAGING: the host pool gets no device staging, so kernel 4 is refused
+    (UNSUPPORTED, nothing enqueued) and the auto choice takes the SM kernel over mapped
+    memory (one launch), byte-exact."""
     case = migration_case("C1", scale=0.25)
     sh = case.shape
     dev, d0 = pool(sh, case.nb_src, 20)
@@ -297,6 +328,10 @@ def test_no_staging_flag_uses_the_sm_path():
     host.tensor().copy_(torch.from_numpy(h0))
     hbt = np.random.default_rng(22).permutation(case.n).astype(np.int32)
     st, ht = dtab(case.src_bt), htab(hbt)
+    with pytest.raises(wk.WindKVError) as e:  # kernel 4 asked for, but no staging: refused
+        wk.swap_out(dev, st, host, ht)
+    assert e.value.status == -10
+    wk.set_tuning(wk.PATH_HOST, kernel=wk.KERNEL_AUTO)
     l0 = wk.launch_count()
     wk.swap_out(dev, st, host, ht)
     torch.cuda.synchronize()

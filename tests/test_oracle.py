@@ -235,6 +235,24 @@ def test_error_precedence():
     assert O.geom_check(O.Geom(0, 0, 1, 16, 1, 1, 1)) == O.INVALID_ARG
 
 
+def test_null_tables_are_invalid_arg_before_geometry_and_layers():
+    """S§8(b) "Errors": INVALID_ARG (every null handle) precedes GEOMETRY and LAYER_RANGE, so a
+    NULL table of a non-empty op is INVALID_ARG even when the pools also mismatch."""
+    import ctypes as ct
+    gs = O.Geom(0, 2, 2, 8, 2, 2, 4)
+    gbad = O.Geom(0, 2, 4, 8, 2, 2, 4)
+    src, dst = rand_pool(gs, 0), rand_pool(gbad, 1)
+    lib = O._lib()
+    for gd, lo, hi in ((gbad, 0, 2), (gs, 0, 9), (gbad, 3, 1)):
+        d = dst if gd is gbad else rand_pool(gs, 2)
+        rc = lib.or_migrate(O._p(src), ct.byref(gs.c()), None, O._p(d), ct.byref(gd.c()),
+                            O._p(np.zeros(1, np.int32)), 1, lo, hi)
+        assert rc == O.INVALID_ARG, (lo, hi, rc)
+    # n == 0 needs no tables: the geometry error stands
+    rc = lib.or_migrate(O._p(src), ct.byref(gs.c()), None, O._p(dst), ct.byref(gbad.c()), None, 0, 0, 2)
+    assert rc == O.GEOMETRY
+
+
 # ---------------------------------------------------------- P5 closed forms / golden
 
 def test_golden_p120_opt13b_bytes():
