@@ -135,3 +135,13 @@ def test_binding_accepts_only_int32_device_accessible_tables():
     with pytest.raises(ValueError):
         wk._ptr(torch.zeros(8, dtype=torch.int32)[::2])  # not contiguous
     assert wk._ptr(None) is None and wk._ptr(1234) == 1234
+
+
+def test_plan_compact_worked_example():
+    """The library's planner on the hand-worked O6 examples (tests/golden/)."""
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "o6_compaction_worked_example.json")))
+    for c in g["cases"]:
+        s, d = wk.plan_compact(np.asarray(c["live"], np.uint8))
+        assert s.tolist() == c["src_bt"] and d.tolist() == c["dst_bt"], c

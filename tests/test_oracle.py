@@ -476,3 +476,17 @@ def test_migrate_heads_errors():
     assert O.check_op_heads(gs, gd, 1, 0, 2, 0, 0, 0) == O.INVALID_ARG
     assert O.check_op_heads(gs, O.Geom(0, 2, 2, 16, 2, 1, 5), 1, 0, 2, 0, 0, 1) == O.GEOMETRY
     assert O.check_op_heads(gs, gd, 1, 0, 3, 0, 0, 1) == O.LAYER_RANGE
+
+
+def test_o6_pairing_worked_example():
+    """O6 pairs holes[k] <- movers[k] (both ascending).  Invariant checks alone accept any
+    valid pairing (e.g. holes ascending <- movers descending); these hand-worked examples
+    (tests/golden/o6_compaction_worked_example.json, S§8(c) O6) pin the pairing itself."""
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "o6_compaction_worked_example.json")))
+    for c in g["cases"]:
+        live = np.asarray(c["live"], np.uint8)
+        assert int(live.sum()) == c["n_live"]
+        s, d = O.plan_compact(live)
+        assert s.tolist() == c["src_bt"] and d.tolist() == c["dst_bt"], c
+        assert c["src_bt"] == c["movers"] and c["dst_bt"] == c["holes"]
