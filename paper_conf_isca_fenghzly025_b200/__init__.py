@@ -167,7 +167,7 @@ def _ptr(x) -> Optional[int]:
             raise TypeError(f"block tables must be int32 tensors, got {x.dtype}")
         if not x.is_contiguous():
             raise ValueError("tables must be contiguous")
-        if not x.is_cuda and not x.is_pinned():
+        if not x.is_cuda and x.numel() > 0 and not x.is_pinned():
             # the kernels read tables on the device: pageable host memory is not accessible
             raise ValueError("block tables must be device tensors or pinned host tensors")
         return x.data_ptr()

@@ -930,7 +930,7 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
   const int32_t lgroups = (hi - lo + lpc - 1) / lpc;
   const int32_t K = lgroups * bchunks;
   // DMA streams: a swap-out alternates chunks over two (two device-to-host copies in flight
-  // drive PCIe ~3.5 % harder than one: 55.9 vs 54.0 GB/s, scripts/ce_parallel_probe.py);
+  // drive PCIe ~3.5 % harder than one: 55.9 vs 54.0 GB/s, round-1 probe);
   // host-to-device gains nothing from a second stream, so a swap-in uses one
   const int nside = (out && K >= 2) ? 2 : 1;
   WKV_CUDA(cudaEventRecord(g.fork, s), "cudaEventRecord(fork)");
