@@ -380,7 +380,20 @@ def run_c5_compaction(wk, device, gpu_index, steps, warmup, barrier=None):
     return pb, ms, int(len(csrc)), gib
 
 
-def run_c1_intra(wk, device, peaks, reps=20, warmup=3) -> dict:
+def run_c1_intra(wk, device, peaks, reps=20, warmup=3, replicas=8) -> dict:
+    """C1 (BJ:configs[0], S§8(d)): the intra-device migrate pool A -> pool B (144 MiB) and the
+    compaction of pool A after freeing half its requests, each measured two ways (the single
+    op is the primary number, as in round 1):
+
+    * single op: one op between two CUDA events with the L2 flushed (read of 2 x L2) before
+      it.  This includes the fixed cost of ANY launch measured this way — an empty kernel
+      between two events after the same flush measures `event_floor_us` (~5 us on B200,
+      profiles/r02/launch_floor_probe.txt) — so a 12 us op can reach at most ~0.7 of HBM.
+    * stream of cold ops: `replicas` independent pool pairs (R x 394 MB >> L2), ops issued
+      back to back round-robin over them, one event pair around K ops: every op reads cold
+      data (its pools were last touched R - 1 ops earlier), and the launch of op k + 1
+      overlaps op k (programmatic dependent launch), as in a serving engine that issues
+      migrations / compactions on a side stream.  Per-op time = window / K."""
     import torch
     from windgen import migration_case, live_mask_after_free, request_lengths, blocks_for_tokens
     dev = torch.device("cuda", device)
@@ -388,11 +401,14 @@ def run_c1_intra(wk, device, peaks, reps=20, warmup=3) -> dict:
     hbm = peaks["hbm_gbs"]
     case = migration_case("C1")
     sh = case.shape
-    a = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
-    b = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag)
+    pairs = [(make_pool(wk, sh, case.nb_src, device, case.content_seed + 100 * r, case.src_tag),
+              make_pool(wk, sh, case.nb_dst, device, case.content_seed + 100 * r, case.dst_tag))
+             for r in range(replicas)]
+    a, b = pairs[0]
     sbt, dbt = torch.as_tensor(case.src_bt, device=dev), torch.as_tensor(case.dst_bt, device=dev)
     l2 = int(getattr(torch.cuda.get_device_properties(device), "L2_cache_size", 0) or (126 << 20))
     flush = torch.ones(2 * l2 // 4, dtype=torch.int32, device=dev)
+    tiny = torch.zeros(1, device=dev)
 
     def timed(fn):
         for _ in range(warmup):
@@ -407,20 +423,42 @@ def run_c1_intra(wk, device, peaks, reps=20, warmup=3) -> dict:
                 e1.record(s)
         torch.cuda.synchronize()
         return float(np.median([e0.elapsed_time(e1) for e0, e1 in ev]))
+
+    def stream_of_ops(op, k=8 * replicas):
+        ms = time_device(lambda: [op(i) for i in range(k)], 3, 1, s) / 3
+        return ms / k
     pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
+    floor_ms = timed(lambda: tiny.add_(0))
     ms = timed(lambda: wk.migrate(a, sbt, b, dbt, stream=s))
+    ms_st = stream_of_ops(lambda i: wk.migrate(pairs[i % replicas][0], sbt, pairs[i % replicas][1], dbt, stream=s))
     res = {"migrate_gbs": round(pb / ms / 1e6, 1), "migrate_hbm_frac": round(2 * pb / ms / 1e6 / hbm, 3),
-           "migrate_ms": round(ms, 4), "payload_mib": round(pb / (1 << 20), 1),
-           "l2_flush_read_bytes_before_each_op": int(flush.numel() * 4)}
+           "migrate_ms": round(ms, 4),
+           "migrate_stream_gbs": round(pb / ms_st / 1e6, 1),
+           "migrate_stream_hbm_frac": round(2 * pb / ms_st / 1e6 / hbm, 3),
+           "migrate_stream_ms_per_op": round(ms_st, 4), "payload_mib": round(pb / (1 << 20), 1),
+           "event_floor_us": round(floor_ms * 1e3, 2),
+           "l2_flush_read_bytes_before_each_single_op": int(flush.numel() * 4),
+           "stream_replicas": replicas,
+           "stream_working_set_mib": round(replicas * (a.nbytes + b.nbytes) / (1 << 20))}
     reqb = blocks_for_tokens(request_lengths("C1"), sh.block_size)
     live, _ = live_mask_after_free(case.nb_src, reqb, 0.5, 4001)
     csrc, cdst = wk.plan_compact(live)
     ts, td = torch.as_tensor(csrc, device=dev), torch.as_tensor(cdst, device=dev)
     pc = payload_bytes(len(csrc), sh.n_layers, sh.chunk_bytes)
     ms = timed(lambda: wk.compact(a, ts, td, stream=s))
+    ms_st = stream_of_ops(lambda i: wk.compact(pairs[i % replicas][0], ts, td, stream=s))
     res.update({"compact_moves": int(len(csrc)), "compact_gbs": round(pc / ms / 1e6, 1),
-                "compact_hbm_frac": round(2 * pc / ms / 1e6 / hbm, 3), "compact_ms": round(ms, 4)})
-    del a, b, flush
+                "compact_hbm_frac": round(2 * pc / ms / 1e6 / hbm, 3), "compact_ms": round(ms, 4),
+                "compact_single_op_ceiling_frac": round(2 * pc / hbm / 1e3 / (2 * pc / hbm / 1e3 + floor_ms * 1e3), 3),
+                "compact_stream_gbs": round(pc / ms_st / 1e6, 1),
+                "compact_stream_hbm_frac": round(2 * pc / ms_st / 1e6 / hbm, 3),
+                "compact_stream_ms_per_op": round(ms_st, 4),
+                "note": "*_hbm_frac / *_ms: one op between CUDA events after an L2 flush; it "
+                        "includes the event_floor_us that an empty launch costs in the same "
+                        "measurement, so compact_single_op_ceiling_frac = ideal / (ideal + floor) "
+                        "bounds it; *_stream_*: ops back to back round-robin over "
+                        "stream_replicas pool pairs (data >> L2), window / ops"})
+    del a, b, pairs, flush
     return res
 
 

@@ -63,6 +63,11 @@ tunings = [("default", None),
            ("simt_u24k_2cta", wk.tuning(kernel=S, stage_bytes=24576, stages=4, ctas_per_sm=2)),
            ("simt_u24k_4cta", wk.tuning(kernel=S, stage_bytes=24576, stages=4, ctas_per_sm=4)),
            ("simt_u48k_4cta", wk.tuning(kernel=S, stage_bytes=49152, stages=4, ctas_per_sm=4))]
+if "--ring" in sys.argv:  # bytes in flight per CTA for small ops (stage x stages, store lag)
+    tunings = [("default", None)] + [
+        (f"tma_u{sb // 1024}k_s{st}_lag{lag}", wk.tuning(kernel=T, stage_bytes=sb, stages=st, store_lag=lag))
+        for sb, st, lag in ((49152, 4, 1), (49152, 4, 3), (32768, 6, 2), (32768, 6, 1),
+                            (24576, 8, 2), (24576, 8, 1), (16384, 12, 3), (16384, 12, 2), (12288, 16, 4))]
 for name, t in tunings:
     r = {}
     for op, fn, by in (("migrate", lambda: wk.migrate_ex(a, sbt, b, dbt, t, stream=s), pb),
@@ -77,6 +82,8 @@ for name, t in tunings:
         if by:
             r[op + "_frac"] = round(2 * by / (us * 1e-6) / 1e9 / hbm, 3)
     # back to back (no flush, no event between): the per-op cost in a stream of ops
+    if len(r) < 5:
+        continue
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with torch.cuda.stream(s):
         ev0.record(s)
