@@ -1,16 +1,29 @@
-# round-end evidence: smoke, GPU suite, default bench, ncu launch list of the default bench
-python -c "import __graft_entry__ as g; g.build(); g.smoke(); print('SMOKE OK')" 2>&1 | tail -2
-mkdir -p gpurun_out
-timeout -s KILL 1500 python -m pytest tests -m gpu -q -x 2>&1 | tail -5 | tee gpurun_out/gpu_tests.log
-timeout -s KILL 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?"
-tail -3 gpurun_out/bench.err
-timeout -s KILL 300 python bench.py --impl reference --steps 3 --warmup 3 > gpurun_out/bench_reference.json 2>&1; echo "ref rc=$?"
+# Round-end evidence on one B200 (run under gpurun): smoke, GPU suite, default bench,
+# reference arm, ncu launch list of the default bench command, ncu --set full on the
+# headline launch, the N>1 bench path with every rank on the one GPU, sanitizers.
+# usage: bash scripts/gpu_final.sh <tag>     (outputs: gpurun_out/<tag>_*)
+T=${1:-r02}
+O=gpurun_out
+mkdir -p $O
+nvidia-smi -L > $O/${T}_smi.txt 2>&1
+timeout -s KILL 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/${T}_smoke.log 2>&1; echo "smoke rc=$?" >> $O/${T}_smoke.log
+timeout -s KILL 1500 python -m pytest tests -m gpu -q > $O/${T}_gputest.log 2>&1; echo "rc=$?" >> $O/${T}_gputest.log
+timeout -s KILL 900 python bench.py > $O/${T}_bench.json 2> $O/${T}_bench.err; echo "bench rc=$?" >> $O/${T}_bench.err
+timeout -s KILL 300 python bench.py --impl reference --steps 3 --warmup 3 > $O/${T}_bench_reference.json 2>&1
 timeout -s KILL 1500 ncu --metrics gpu__time_duration.sum --clock-control none -c 2500 --csv \
-   --log-file gpurun_out/launches_final.csv python bench.py --steps 5 --warmup 3 --no-cpu-baseline \
-   > gpurun_out/launches_bench_final.json 2>&1
-echo "launches rc=$?"
+   --log-file $O/${T}_launches.csv python bench.py --steps 5 --warmup 3 --no-cpu-baseline \
+   > $O/${T}_launches_bench.json 2>&1; echo "launches rc=$?" >> $O/${T}_bench.err
 # full section set on the headline launch (application replay: the pools are ~95 GiB)
 timeout -s KILL 1500 ncu --set full --clock-control none --import-source on --replay-mode application \
-   -k regex:tma_copy -s 3 -c 1 -o gpurun_out/prof_tma_c2_final \
-   python bench.py --steps 1 --warmup 3 --no-scenarios --no-cpu-baseline > gpurun_out/prof_bench_final.json 2>&1
-echo "full rc=$?"
+   -k regex:tma_copy -s 3 -c 1 -o $O/${T}_prof_tma_c2 \
+   python bench.py --steps 1 --warmup 3 --no-scenarios --no-cpu-baseline > $O/${T}_prof_bench.json 2>&1
+echo "full rc=$?" >> $O/${T}_bench.err
+# the N>1 path (pairs over CUDA IPC, all-to-all batch pushes) with every rank on this GPU:
+# a functional check only, NOT multi-GPU bandwidth
+export WIND_BENCH_ONE_DEVICE=1
+timeout -s KILL 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 \
+  --master-port 29533 bench.py --gpus 2 --steps 5 --warmup 3 --a2a-scale 0.125 --config C1 \
+  > $O/${T}_multirank2.log 2>&1; echo "multirank2 rc=$?" >> $O/${T}_multirank2.log
+unset WIND_BENCH_ONE_DEVICE
+bash scripts/sanitize.sh > $O/${T}_sanitize_summary.txt 2>&1
+ls -la $O > $O/${T}_ls.txt
