@@ -1129,9 +1129,15 @@ def run_gpu(args) -> None:
         # a failure prints one explanatory line instead of a traceback and a hung barrier
         err = None
         try:
-            handles = parallel.exchange_handles(dst.export() if role == "decode" else None)
+            # both pools of a pair are exported: the push rank imports the decode pool (push:
+            # the prefill GPU's SMs store over NVLink), the decode rank imports the prefill
+            # pool (pull: the decode GPU's SMs load over NVLink) — the autotune below times both
+            handles = parallel.exchange_handles(dst.export() if role == "decode" else
+                                                (src.export() if role == "push" else None))
             if role == "push":
                 dst = wk.Pool.import_(handles[partner], local)
+            elif role == "decode":
+                src = wk.Pool.import_(handles[partner], local)
         except Exception as e:  # noqa: BLE001 — reported below, then the run ends
             err = f"rank {rank}: {type(e).__name__}: {e}"[:300]
         errs: list = [None] * world
@@ -1150,8 +1156,15 @@ def run_gpu(args) -> None:
     lo, hi = 0, sh.n_layers
     pb = payload_bytes(case.n, hi - lo, sh.chunk_bytes)
 
+    # who executes a pair's op: "push" = the prefill rank (src local, dst imported), "pull" =
+    # the decode rank (src imported, dst local); a solo rank always runs its own op
+    mode = {"v": "push"}
+
+    def executes() -> bool:
+        return role == "solo" or (role == "push") == (mode["v"] == "push")
+
     def step():
-        if role != "decode":
+        if executes():
             wk.migrate(src, sbt, dst, dbt, layer_lo=lo, layer_hi=hi, stream=stream)
 
     # N > 1: the peer-path kernel is chosen on the real link before the timed steps (round 1
@@ -1160,24 +1173,29 @@ def run_gpu(args) -> None:
     # PEER tuning for the headline.  Reported as `peer_autotune` in the line.
     peer_tune = None
     if world > 1:
-        cands = [("simt_96ctas", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=32768, stages=6,
-                                       max_ctas=96)),
-                 ("simt_4x148", dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768, stages=6)),
-                 ("tma_148", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, store_lag=2)),
-                 ("tma_64", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, store_lag=2,
-                                 max_ctas=64)),
-                 ("tma_32", dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, store_lag=2,
-                                 max_ctas=32))]
+        simt96 = dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=1, stage_bytes=32768, stages=6, max_ctas=96)
+        simt4 = dict(kernel=wk.KERNEL_SIMT, ctas_per_sm=4, stage_bytes=32768, stages=6)
+        tma148 = dict(kernel=wk.KERNEL_TMA, ctas_per_sm=1, stage_bytes=49152, stages=4, store_lag=2)
+        cands = [("push_simt_96ctas", "push", simt96), ("push_simt_4x148", "push", simt4),
+                 ("push_tma_148", "push", tma148), ("push_tma_64", "push", {**tma148, "max_ctas": 64}),
+                 ("push_tma_32", "push", {**tma148, "max_ctas": 32}),
+                 ("pull_simt_4x148", "pull", simt4), ("pull_tma_148", "pull", tma148),
+                 ("pull_tma_64", "pull", {**tma148, "max_ctas": 64})]
+        default_peer = wk.get_tuning(wk.PATH_PEER)
         try:
             rates = {}
-            for name, cfg in cands:
+            for name, m, cfg in cands:
+                mode["v"] = m
                 wk.set_tuning(wk.PATH_PEER, **cfg)
                 ms_alt, = parallel.max_over_ranks([time_device(step, 3, 3, stream, barrier) / 3])
                 rates[name] = round(pb / ms_alt / 1e6, 1)
             best = max(rates, key=rates.get)
-            wk.set_tuning(wk.PATH_PEER, **dict(cands)[best])
+            _, mode["v"], cfg = next(c for c in cands if c[0] == best)
+            wk.set_tuning(wk.PATH_PEER, **cfg)
             peer_tune = {"chosen": best, "gbs_per_pair": rates}
-        except Exception as e:  # noqa: BLE001 — reported; the library default stays
+        except Exception as e:  # noqa: BLE001 — reported; the library default (push) stays
+            mode["v"] = "push"
+            wk.set_tuning(wk.PATH_PEER, **default_peer)
             peer_tune = {"error": f"{type(e).__name__}: {e}"[:300]}
             print(f"[bench rank {rank}] peer autotune failed: {peer_tune['error']}", file=sys.stderr, flush=True)
     torch.cuda.synchronize()
@@ -1185,7 +1203,11 @@ def run_gpu(args) -> None:
     step_ms: list = []
     with ClockSampler(local) as clk:
         ms_total = time_device(step, args.steps, args.warmup, stream, barrier, per_step=step_ms)
-    launches = wk.launch_count() - launches0 - (args.warmup if role != "decode" else 0)
+    launches = wk.launch_count() - launches0 - (args.warmup if executes() else 0)
+    if world > 1:  # every rank's library launches in the timed region (pull: the decode ranks')
+        t_l = torch.tensor([float(launches)], dtype=torch.float64)
+        dist.all_reduce(t_l)
+        launches = int(t_l.item())
     ms_step_local = ms_total / args.steps
     # e2e: tables from pinned host memory H2D, the migrate, the layer flags read back D2H
     h_sbt = torch.as_tensor(case.src_bt).pin_memory()
@@ -1194,7 +1216,7 @@ def run_gpu(args) -> None:
     flags_host = torch.empty(sh.n_layers, dtype=torch.int32).pin_memory()
 
     def e2e_step():
-        if role == "decode":
+        if not executes():
             return
         with torch.cuda.stream(stream):
             d_sbt.copy_(h_sbt, non_blocking=True)
@@ -1236,7 +1258,7 @@ def run_gpu(args) -> None:
 
     extra = {}
     if rank == 0:
-        kernel_gbs = pb / ms_step_local / 1e6
+        kernel_gbs = pb / ms_step / 1e6  # one mover's op (max over ranks: the executing rank)
         if role == "solo":
             roof = {"bound": "hbm", "achieved": round(2 * kernel_gbs, 1), "peak": peaks["hbm_gbs"],
                     "unit": "GB/s", "frac": round(2 * kernel_gbs / peaks["hbm_gbs"], 4),
@@ -1276,7 +1298,10 @@ def run_gpu(args) -> None:
                                    f"requests ({LENGTH_MIX.get(args.config, '')}), {args.variant} tables, "
                                    f"prefill pool -> decode pool, layers 0-{sh.n_layers - 1}",
                        "payload_gib_per_pair": round(pb / GiB, 3),
-                       "placement": "same GPU" if world == 1 else "pairs 2k->2k+1 over NVLink peer stores",
+                       "placement": "same GPU" if world == 1 else (
+                           "pairs 2k->2k+1 over NVLink, " + ("push: the prefill GPU stores into the peer pool"
+                                                              if mode["v"] == "push" else
+                                                              "pull: the decode GPU loads from the peer pool")),
                        "l2": "inputs >> 126 MB L2 (no flush needed)",
                        "parallelism": f"{n_movers} independent mover(s)", "seed_offset": args.seed},
             "e2e": {"value": round(e2e_value, 2), "unit": "GB/s",
