@@ -863,6 +863,11 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         [(f"cap{c or 'none'}", {**saved, "max_ctas": c}) for c in (2, 4, 8, 16, 0)] +
         [(f"rate{r}GBs", {**saved, "max_ctas": 0, "rate_mbps": r * 1000}) for r in (50, 100, 150, 300)] +
         [(f"rate{r}GBs_32ctas", {**saved, "max_ctas": 32, "rate_mbps": r * 1000}) for r in (100,)] +
+        # L2 evict-first on the migration's loads and stores: the streamed KV should not push
+        # the victim's small hot data (block tables, queries, partial outputs) out of L2
+        [(f"rate{r}GBs_evict_first", {**saved, "max_ctas": 0, "rate_mbps": r * 1000, "evict_first": 1})
+         for r in (50, 150)] +
+        [("cap2_evict_first", {**saved, "max_ctas": 2, "evict_first": 1})] +
         [(f"copy_engines_rate{r}GBs", {**saved, "kernel": wk.KERNEL_COPY_ENGINE, "rate_mbps": r * 1000})
          for r in (50, 100, 150, 300)] +
         # SM partition (green contexts, wind_kv_partition_sms): migration confined to 8 SMs,
