@@ -1,0 +1,20 @@
+"""Development helper: one bench.py scenario alone, printed as one JSON line.
+usage: python scripts/run_part.py c1_intra|interference|handoff|stall_free|pressure|next3|policy"""
+import json
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import bench  # noqa: E402
+import paper_conf_isca_fenghzly025_b200 as wk  # noqa: E402
+
+peaks = bench.load_peaks()
+name = sys.argv[1]
+fn = {"c1_intra": lambda: bench.run_c1_intra(wk, 0, peaks),
+      "interference": lambda: bench.run_interference(wk, 0, peaks),
+      "handoff": lambda: bench.run_handoff(wk, 0),
+      "stall_free": lambda: bench.run_stall_free(wk, 0),
+      "pressure": lambda: bench.run_pressure(wk, 0),
+      "next3": lambda: bench.run_next3(wk, 0, peaks),
+      "policy": lambda: bench.run_policy_profile(wk, 0)}[name]
+print(json.dumps({name: fn()}))
