@@ -1299,9 +1299,7 @@ def run_gpu(args) -> None:
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_step, 4),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
             "dtype": "u8", "data": "synthetic",
-            "config": {"workload": f"{args.config} {sh.name} KV: {case.n} blocks of {case.lengths.size} "
-                                   f"requests ({LENGTH_MIX.get(args.config, '')}), {args.variant} tables, "
-                                   f"prefill pool -> decode pool, layers 0-{sh.n_layers - 1}",
+            "config": {"workload": workload_name(args, case),
                        "payload_gib_per_pair": round(pb / GiB, 3),
                        "placement": "same GPU" if world == 1 else (
                            "pairs 2k->2k+1 over NVLink, " + ("push: the prefill GPU stores into the peer pool"
@@ -1340,6 +1338,14 @@ def traffic_from_profiles(cfg: str):
         return None
 
 
+def workload_name(args, case) -> str:
+    """config.workload of both arms (the wind_kv line and --impl reference)."""
+    sh = case.shape
+    return (f"{args.config} {sh.name} KV: {case.n} blocks of {case.lengths.size} "
+            f"requests ({LENGTH_MIX.get(args.config, '')}), {args.variant} tables, "
+            f"prefill pool -> decode pool, layers 0-{sh.n_layers - 1}")
+
+
 def run_reference(args) -> None:
     """--impl reference: the CPU oracle as it stands on this host's cores, rank 0 only."""
     rank = int(os.environ.get("RANK", 0))
@@ -1371,7 +1377,7 @@ def run_reference(args) -> None:
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
         "ms_per_step": round(el / args.steps * 1e3, 3), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic",
-        "config": {"workload": f"{args.config} {sh.name} KV, {args.variant} tables (oracle sample)"},
+        "config": {"workload": workload_name(args, case), "sample": "oracle on host cores, bounded sample: " + sample},
         "cpu_baseline": {"value": round(v, 3), "unit": "GB/s", "cores": T, "kind": "oracle",
                          "sample": sample},
         "e2e": {"value": round(v, 3), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
