@@ -37,6 +37,8 @@
  *     serialization must call cudaGridDependencySynchronize() before reading the op's
  *     destination (the standard PDL contract).  WIND_KV_PDL=0 in the environment turns it
  *     off.
+ *   - WIND_KV_FORCE_SYS_SCOPE=1 in the environment (tests): every op publishes its layer
+ *     flags at system scope, as peer destinations always do (wind_kv_route reports it).
  */
 #ifndef WIND_KV_H
 #define WIND_KV_H

@@ -173,6 +173,17 @@ bool blocked_dealing_enabled() {
   }();
   return on;
 }
+// WIND_KV_FORCE_SYS_SCOPE=1 publishes every op's layer flags at system scope, as a peer
+// (NVLink) destination requires: lets one-GPU tests run the peer publication path (the
+// fences, the .sys reductions on device-memory flags) with the data on one device.
+bool force_sys_scope() {
+  static const bool on = [] {
+    const char* e = getenv("WIND_KV_FORCE_SYS_SCOPE");
+    return e && e[0] == '1';
+  }();
+  return on;
+}
+
 constexpr int kHostCtasFromHost = 8;
 constexpr int64_t kStagedInFlight = 768 << 10;
 
@@ -1148,7 +1159,8 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     q.host_flags = d->desc.loc == WIND_LOC_HOST;
     // GPU-scope publication only when both pools live on the executing GPU (same physical
     // device: every reader of the data and of the flags goes through this GPU's L2)
-    q.sys_scope = !(src->desc.loc == WIND_LOC_DEVICE && d->desc.loc == WIND_LOC_DEVICE &&
+    q.sys_scope = force_sys_scope() ||
+                  !(src->desc.loc == WIND_LOC_DEVICE && d->desc.loc == WIND_LOC_DEVICE &&
                     memcmp(src->uuid, d->uuid, 16) == 0);
     p.sys_scope |= q.sys_scope;
     const int64_t u = p.parts > 1 ? static_cast<int64_t>(it.n) * p.parts
@@ -1288,7 +1300,8 @@ extern "C" wind_status wind_kv_route(const wind_kv_pool* src, const wind_kv_pool
   // the publication scope run_op chooses: GPU scope only when both pools are device pools on
   // the executing GPU
   if (sys_scope)
-    *sys_scope = !(src->desc.loc == WIND_LOC_DEVICE && dst->desc.loc == WIND_LOC_DEVICE &&
+    *sys_scope = force_sys_scope() ||
+                 !(src->desc.loc == WIND_LOC_DEVICE && dst->desc.loc == WIND_LOC_DEVICE &&
                    memcmp(src->uuid, dst->uuid, 16) == 0);
   return WIND_OK;
 }
