@@ -670,6 +670,17 @@ def run_pressure(wk, device, reps: int = 3) -> dict:
     t_x = time_device(exchange, reps, 1, s_mig) / reps
     out["swap_exchange"] = {"ms": round(t_x, 2), "aggregate_gbs": round(2 * vb / t_x / 1e6, 1),
                             "note": "swap-out and swap-in of 12.7 GiB each at the same time (default SM paths)"}
+    # the same eviction and exchange through the opt-in staged copy-engine path (kernel 4:
+    # host tables read on the CPU at enqueue; the pinned host-slot table ht_h)
+    saved_h = wk.get_tuning(wk.PATH_HOST)
+    wk.set_tuning(wk.PATH_HOST, **{**saved_h, "kernel": wk.KERNEL_STAGED})
+    try:
+        t_sw_st = time_device(lambda: wk.swap_out(dpool, vt, host, ht_h, stream=s_swap), reps, 1, s_swap) / reps
+        t_x_st = time_device(exchange, reps, 1, s_mig) / reps
+    finally:
+        wk.set_tuning(wk.PATH_HOST, **saved_h)
+    out["staged_opt_in"] = {"swap_gbs": round(vb / t_sw_st / 1e6, 1),
+                            "swap_exchange_aggregate_gbs": round(2 * vb / t_x_st / 1e6, 1)}
     host2.destroy()
     del dpool, host, other, src_inc
     return out
