@@ -265,6 +265,42 @@ def test_invalid_arg_precedes_geometry_and_layer_range():
     torch.cuda.synchronize()
 
 
+def test_argument_precedence_random_vs_oracle():
+    """300 random argument combinations (NULL tables, n < 0 / 0 / > 0, same-geometry /
+    other-H / same pool, layer windows in and out of range, inverted and empty ranges): the
+    library's status equals the oracle's (or_migrate, which states S§8(b)'s precedence)."""
+    import ctypes as ct
+    sh = KVShape("t", 4, 2, 64, 2)
+    a, a0 = make_pool(sh, 6, 1)
+    b, b0 = make_pool(sh, 6, 2, first_layer=2)
+    c = wk.Pool(4, 4, 64, 16, 2, 6)  # different H
+    c0 = np.zeros(c.nbytes, np.uint8)
+    host = {id(a): a0, id(b): b0, id(c): c0}
+    sbt_d, dbt_d = tab([0, 1]), tab([2, 3])
+    sbt_h, dbt_h = np.array([0, 1], np.int32), np.array([2, 3], np.int32)
+    lib = O._lib()
+    rng = np.random.default_rng(77)
+    seen = set()
+    for _ in range(300):
+        dst = [a, b, c][int(rng.integers(0, 3))]
+        n = int(rng.choice([-1, 0, 1, 2]))
+        null_s, null_d = bool(rng.random() < 0.25), bool(rng.random() < 0.25)
+        lo = int(rng.integers(-1, 8))
+        hi = int(rng.integers(-1, 8))
+        got = status_of(wk.migrate, a, None if null_s else sbt_d.data_ptr(), dst,
+                        None if null_d else dbt_d.data_ptr(), n=n, layer_lo=lo, layer_hi=hi)
+        src_h = host[id(a)]
+        dst_h = src_h if dst is a else host[id(dst)].copy()
+        want = lib.or_migrate(O._p(src_h), ct.byref(geom(a).c()),
+                              None if null_s else O._p(sbt_h), O._p(dst_h), ct.byref(geom(dst).c()),
+                              None if null_d else O._p(dbt_h), n, lo, hi)
+        assert got == want, dict(dst="abc"[[a, b, c].index(dst)], n=n, null=(null_s, null_d), lo=lo, hi=hi,
+                                 got=got, want=want)
+        seen.add(got)
+    assert {0, -1, -2, -3} <= seen  # every precedence class was exercised
+    torch.cuda.synchronize()
+
+
 def test_wrong_device_stream_precedes_geometry():
     """A stream of another device is INVALID_ARG even when the pools also mismatch (needs
     two GPUs to build such a stream)."""
