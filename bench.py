@@ -776,13 +776,19 @@ def run_stall_free(wk, device, cap_ctas: int = 16) -> dict:
     theta = stall_free.default_theta(max(step_ms, 0.05), bw, sh.n_layers, sh.chunk_bytes)
     res = stall_free.migrate_stall_free(src, st, dst, dt, T0, theta, step, mig, dec)
     wk.set_tuning(wk.PATH_INTRA, **saved)
+    # the same request with its stages issued as full-rate bursts of 8 blocks (100 MiB) per
+    # decode step (chunk_blocks; the interference rows show why: burst vs trickle)
+    resb = stall_free.migrate_stall_free(src, st, dst, dt, T0 + 64, theta, step, mig, dec, chunk_blocks=8)
     del src, dst
     return {"request": "OPT-13B, 2048 tokens at start (P:120)", "cap_ctas": cap_ctas,
             "migration_gbs": round(bw, 1), "stop_the_world_ms": round(stw, 3),
             "theta_blocks": theta, "stages": len(res.stages), "tokens_decoded_while_migrating":
             int(sum(res.appends)), "pause_ms": round(res.pause_ms, 3),
             "blocked_time_reduction": round(1 - res.pause_ms / stw, 4),
-            "blocks_sent": res.blocks_sent}
+            "blocks_sent": res.blocks_sent,
+            "bursts_of_8_blocks_per_decode_step": {
+                "stages": len(resb.stages), "tokens_decoded_while_migrating": int(sum(resb.appends)),
+                "pause_ms": round(resb.pause_ms, 3), "blocks_sent": resb.blocks_sent}}
 
 
 def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict:
@@ -1025,6 +1031,46 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             res[name].update({"partition_sms_migration": P.sms_migration, "partition_sms_compute": P.sms_compute,
                               "victim_ms_alone_whole_gpu": round(t_full, 3),
                               "slowdown_vs_whole_gpu": round(t_with / t_full - 1.0, 4)})
+    # Burst instead of trickle: the same AVERAGE migration rate delivered as one full-rate op
+    # per decode step, released by an event at the step's start (the op overlaps the first
+    # part of the step), against the rate-limited trickle rows above.  A trickle holds HBM
+    # (and SMs) for the whole step; a burst finishes early and leaves the rest of the step
+    # alone, so the victim's added time per migrated byte can differ.
+    wk.set_tuning(wk.PATH_INTRA, **saved)
+    blk_bytes = payload_bytes(1, sh.n_layers, sh.chunk_bytes)
+    for avg in (50, 150, 300):
+        nb_step = max(1, min(case.n, round(avg * 1e9 * t_alone * 1e-3 / blk_bytes)))
+        sb_, db_ = d_tabs[0][:nb_step], d_tabs[1][:nb_step]
+        t_b = time_device(lambda: wk.migrate(src, sb_, dst, db_, n=nb_step, stream=lo_s), 3, 2, lo_s) / 3
+
+        def burst_run(n):
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
+            ev[0].record(hi_s)
+            for i in range(n):
+                go = torch.cuda.Event()
+                go.record(hi_s)
+                lo_s.wait_event(go)
+                wk.migrate(src, sb_, dst, db_, n=nb_step, stream=lo_s)
+                with torch.cuda.stream(hi_s):
+                    graph.replay()
+                ev[i + 1].record(hi_s)
+            return ev
+        alone_b, with_b = [], []
+        for _ in range(rounds):
+            torch.cuda.synchronize()
+            ev = victim_run(n_round)
+            torch.cuda.synchronize()
+            alone_b += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
+            ev = burst_run(n_round)
+            torch.cuda.synchronize()
+            with_b += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
+        tr, tw = float(np.median(alone_b)), float(np.median(with_b))
+        res[f"burst_avg{avg}GBs"] = {
+            "blocks_per_step": int(nb_step), "mb_per_step": round(nb_step * blk_bytes / 1e6, 1),
+            "avg_gbs": round(nb_step * blk_bytes / tr / 1e6, 1), "burst_ms_alone": round(t_b, 3),
+            "victim_ms_alone_adjacent": round(tr, 3), "victim_ms_with_migration": round(tw, 3),
+            "slowdown": round(tw / tr - 1.0, 4),
+            "note": "one full-rate op per decode step, released at the step's start"}
     clk.__exit__()
     wk.set_tuning(wk.PATH_INTRA, **saved)
     wk.set_tuning(wk.PATH_HOST, **saved_host)

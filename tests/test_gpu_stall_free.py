@@ -18,10 +18,11 @@ pytestmark = pytest.mark.gpu
 DEV = torch.device("cuda", 0)
 
 
-@pytest.mark.parametrize("theta,cap", [(2, 2), (1, 4), (8, 0)])
-def test_stall_free_migration_matches_oracle(theta, cap):
+@pytest.mark.parametrize("theta,cap,chunk", [(2, 2, 0), (1, 4, 0), (8, 0, 0), (2, 0, 8), (1, 0, 3)])
+def test_stall_free_migration_matches_oracle(theta, cap, chunk):
     """P:120's request: OPT-13B KV, 2048 tokens (1.5625 GiB).  The migration is throttled
-    (CTA cap) so the request decodes through several stages."""
+    (CTA cap) so the request decodes through several stages; with `chunk`, each stage is
+    issued as one burst of `chunk` blocks per decode step (full rate)."""
     sh = SHAPES["C2"]
     bs = sh.block_size
     T0 = 2048 - 37
@@ -45,7 +46,7 @@ def test_stall_free_migration_matches_oracle(theta, cap):
         dt = torch.as_tensor(dst_slots, device=DEV)
         step(T0)  # warm the append kernel (idempotent: the same bytes are written again later)
         torch.cuda.synchronize()
-        res = stall_free.migrate_stall_free(src, st, dst, dt, T0, theta, step, mig, dec)
+        res = stall_free.migrate_stall_free(src, st, dst, dt, T0, theta, step, mig, dec, chunk_blocks=chunk)
     finally:
         wk.set_tuning(wk.PATH_INTRA, **saved)
     torch.cuda.synchronize()
@@ -70,5 +71,8 @@ def test_stall_free_migration_matches_oracle(theta, cap):
     # the last block sent holds tokens written after T0
     assert sum(res.appends) > 0
     assert all(dst.layer_count(l) == res.ticket for l in range(sh.n_layers))
-    if theta < 8:
-        assert len(res.stages) >= 3
+    if theta < 8:  # capped: the request outgrows theta during stage 0; bursts: at least one stage + pause
+        assert len(res.stages) >= (2 if chunk else 3)
+    if chunk:  # every pre-pause stage took at least one decode step per burst
+        for (b, e), a in zip(res.stages[:-1], res.appends):
+            assert a >= -(-(e - b) // chunk)
