@@ -875,6 +875,11 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     sw_dev = torch.as_tensor(case.src_bt[:n_sw], device=dev)
     sw_host = {"dev": torch.arange(n_sw, dtype=torch.int32, device=dev),
                "pinned": torch.arange(n_sw, dtype=torch.int32).pin_memory()}
+    # push-source proxy: a 1-block destination pool (36 MiB, L2-resident); its table maps
+    # every source block to slot 0 — duplicate destinations, outside the table contract on
+    # purpose (the bytes are never read; release builds do not check table content)
+    sink = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, 1, device=device)
+    zeros_t = torch.zeros(case.n, dtype=torch.int32, device=dev)
     configs = configs or (
         [("control_no_migration", {**saved, "null_feeder": True})] +
         [(f"cap{c or 'none'}", {**saved, "max_ctas": c}) for c in (2, 4, 8, 16, 0)] +
@@ -900,7 +905,15 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
          ("swap_out_sm_8ctas", {"op": "swap_out", **saved_host, "kernel": wk.KERNEL_TMA, "max_ctas": 8}),
          ("swap_in_sm_default", {"op": "swap_in", **saved_host, "kernel": wk.KERNEL_TMA}),
          ("swap_out_staged", {"op": "swap_out", **saved_host, "kernel": wk.KERNEL_STAGED}),
-         ("swap_in_staged", {"op": "swap_in", **saved_host, "kernel": wk.KERNEL_STAGED})])
+         ("swap_in_staged", {"op": "swap_in", **saved_host, "kernel": wk.KERNEL_STAGED})] +
+        # SOURCE side of an NVLink push, emulated on one GPU: the migration reads its source
+        # blocks from this HBM at the link's rate, and its stores all land in ONE destination
+        # block (36 MiB over all layers: they stay in L2), so this HBM sees the push's reads
+        # and almost none of its writes — what a prefill GPU pushing to a peer sees.  A proxy
+        # (no NVLink traffic, the source-side HBM load only), labelled as such.
+        [(f"push_source_proxy_rate{r}GBs", {**saved, "op": "push_source_proxy", "max_ctas": 0,
+                                            "rate_mbps": r * 1000}) for r in (350, 700)] +
+        [("push_source_proxy_uncapped", {**saved, "op": "push_source_proxy", "max_ctas": 0})])
     rounds, n_round = 3, max(10, n_victim_steps // 2)
     part = {}  # SM partition (green contexts): victim graph on the compute SMs
     clk = ClockSampler(device).__enter__()  # SM clock / power per phase (power-cap effects)
@@ -936,6 +949,12 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
 
             def one_op():
                 wk.migrate(src, sbt, dst, dbt, n=case.n, stream=mig_s)
+        elif op_kind == "push_source_proxy":
+            wk.set_tuning(wk.PATH_INTRA, **cfg)
+            op_bytes = pb
+
+            def one_op():  # every source block -> destination block 0 (stays in L2)
+                wk.migrate(src, d_tabs[0], sink, zeros_t, n=case.n, stream=mig_s)
         else:
             wk.set_tuning(wk.PATH_HOST, **cfg)
             ht = sw_host["pinned" if cfg.get("kernel") == wk.KERNEL_STAGED else "dev"]
@@ -1001,7 +1020,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
         t_ref, t_with = float(np.median(alone_all)), float(np.median(with_all))
         # HBM bytes per payload byte: intra-device read + write; SM swap one way; the staged
         # swap adds its gather / scatter through the staging buffer (3 ways)
-        hbm_ways = 2 if op_kind == "migrate" else (3 if cfg.get("kernel") == wk.KERNEL_STAGED else 1)
+        hbm_ways = 2 if op_kind == "migrate" else (3 if cfg.get("kernel") == wk.KERNEL_STAGED else 1)  # proxy: reads
         res[name] = {
             "migration_gbs_alone": round(op_bytes / t_mig / 1e6, 1),
             "migration_hbm_share": round(hbm_ways * op_bytes / t_mig / 1e6 / peaks["hbm_gbs"], 4),
@@ -1038,10 +1057,11 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     # alone, so the victim's added time per migrated byte can differ.
     wk.set_tuning(wk.PATH_INTRA, **saved)
     blk_bytes = payload_bytes(1, sh.n_layers, sh.chunk_bytes)
-    for avg in (50, 150, 300):
+    for avg, proxy in ((50, False), (150, False), (300, False), (700, True)):
         nb_step = max(1, min(case.n, round(avg * 1e9 * t_alone * 1e-3 / blk_bytes)))
-        sb_, db_ = d_tabs[0][:nb_step], d_tabs[1][:nb_step]
-        t_b = time_device(lambda: wk.migrate(src, sb_, dst, db_, n=nb_step, stream=lo_s), 3, 2, lo_s) / 3
+        sb_ = d_tabs[0][:nb_step]
+        db_, dpool_ = (zeros_t[:nb_step], sink) if proxy else (d_tabs[1][:nb_step], dst)
+        t_b = time_device(lambda: wk.migrate(src, sb_, dpool_, db_, n=nb_step, stream=lo_s), 3, 2, lo_s) / 3
 
         def burst_run(n):
             ev = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
@@ -1050,7 +1070,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
                 go = torch.cuda.Event()
                 go.record(hi_s)
                 lo_s.wait_event(go)
-                wk.migrate(src, sb_, dst, db_, n=nb_step, stream=lo_s)
+                wk.migrate(src, sb_, dpool_, db_, n=nb_step, stream=lo_s)
                 with torch.cuda.stream(hi_s):
                     graph.replay()
                 ev[i + 1].record(hi_s)
@@ -1065,7 +1085,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
             torch.cuda.synchronize()
             with_b += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
         tr, tw = float(np.median(alone_b)), float(np.median(with_b))
-        res[f"burst_avg{avg}GBs"] = {
+        res[f"burst_{'push_source_proxy_' if proxy else ''}avg{avg}GBs"] = {
             "blocks_per_step": int(nb_step), "mb_per_step": round(nb_step * blk_bytes / 1e6, 1),
             "avg_gbs": round(nb_step * blk_bytes / tr / 1e6, 1), "burst_ms_alone": round(t_b, 3),
             "victim_ms_alone_adjacent": round(tr, 3), "victim_ms_with_migration": round(tw, 3),
@@ -1078,7 +1098,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     for P, _ in part.values():
         P.destroy()
     host.destroy()
-    del vpool, src, dst
+    del vpool, src, dst, sink
     return res
 
 

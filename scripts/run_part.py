@@ -1,5 +1,5 @@
 """Development helper: one bench.py scenario alone, printed as one JSON line.
-usage: python scripts/run_part.py c1_intra|interference|burst|handoff|stall_free|pressure|next3|policy"""
+usage: python scripts/run_part.py c1_intra|interference|burst|proxy|handoff|stall_free|pressure|next3|policy"""
 import json
 import os
 import sys
@@ -16,6 +16,11 @@ fn = {"c1_intra": lambda: bench.run_c1_intra(wk, 0, peaks),
       "burst": lambda: bench.run_interference(wk, 0, peaks, configs=[
           (f"rate{r}GBs", {**wk.get_tuning(wk.PATH_INTRA), "max_ctas": 0, "rate_mbps": r * 1000})
           for r in (50, 150)]),
+      "proxy": lambda: bench.run_interference(wk, 0, peaks, configs=[
+          (f"push_source_proxy_rate{r}GBs", {**wk.get_tuning(wk.PATH_INTRA), "op": "push_source_proxy",
+                                              "max_ctas": 0, "rate_mbps": r * 1000}) for r in (350, 700)] + [
+          ("push_source_proxy_uncapped", {**wk.get_tuning(wk.PATH_INTRA), "op": "push_source_proxy",
+                                          "max_ctas": 0})]),
       "handoff": lambda: bench.run_handoff(wk, 0),
       "stall_free": lambda: bench.run_stall_free(wk, 0),
       "pressure": lambda: bench.run_pressure(wk, 0),
