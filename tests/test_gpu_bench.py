@@ -48,6 +48,8 @@ def test_bench_multirank_on_one_gpu(world):
     out = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
     assert out.returncode == 0, (out.stdout[-2000:], out.stderr[-3000:])
     d = _json_line(out.stdout)
-    assert d["n_gpus"] == world and d["value"] > 0 and d["gpu_launches"] == 3
+    # launches summed over ranks: one per step per mover (pairs + an unpaired last rank)
+    assert d["n_gpus"] == world and d["value"] > 0 and d["gpu_launches"] == 3 * (world // 2 + world % 2)
+    assert d["peer_autotune"].get("chosen", "").split("_")[0] in ("push", "pull"), d["peer_autotune"]
     a2a = d["scenarios"]["c5_all_to_all"]
     assert a2a["shuffle"]["blocks_moved"] > 0 and a2a["rebalance"]["aggregate_gbs"] >= 0
