@@ -39,6 +39,9 @@
  *     off.
  *   - WIND_KV_FORCE_SYS_SCOPE=1 in the environment (tests): every op publishes its layer
  *     flags at system scope, as peer destinations always do (wind_kv_route reports it).
+ *     WIND_KV_FORCE_PEER_ROUTE=1 (tests): an op between a local pool and a pool imported
+ *     from another process on the SAME GPU takes the PEER route (PEER tuning, system scope),
+ *     so one-GPU runs exercise the multi-GPU path's choices.
  */
 #ifndef WIND_KV_H
 #define WIND_KV_H

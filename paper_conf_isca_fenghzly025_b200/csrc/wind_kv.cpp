@@ -184,6 +184,18 @@ bool force_sys_scope() {
   return on;
 }
 
+// WIND_KV_FORCE_PEER_ROUTE=1 routes an op between this process's pool and an IMPORTED pool
+// of the same physical GPU (another process's pool, as under the N > 1 bench with every
+// rank on one GPU) as a PEER op: the PEER tuning and system-scope publication, so one-GPU
+// runs exercise the multi-GPU bench's peer-path choices.  Off by default.
+bool force_peer_route() {
+  static const bool on = [] {
+    const char* e = getenv("WIND_KV_FORCE_PEER_ROUTE");
+    return e && e[0] == '1';
+  }();
+  return on;
+}
+
 constexpr int kHostCtasFromHost = 8;
 constexpr int64_t kStagedInFlight = 768 << 10;
 
@@ -690,6 +702,13 @@ int exec_device_of(const wind_kv_pool* src, const wind_kv_pool* dst) {
   return -1;
 }
 
+// Both pools are device pools whose data and flags every reader reaches through the
+// executing GPU's L2 (same physical GPU), and the op is not forced onto the peer route.
+bool local_pair(const wind_kv_pool* a, const wind_kv_pool* b) {
+  return a->desc.loc == WIND_LOC_DEVICE && b->desc.loc == WIND_LOC_DEVICE &&
+         memcmp(a->uuid, b->uuid, 16) == 0 && !(force_peer_route() && (a->imported || b->imported));
+}
+
 // Which device runs the op, and which tuning path applies.
 wind_status route(const wind_kv_pool* src, const wind_kv_pool* dst, int* exec, int* path) {
   const bool sd = src->desc.loc == WIND_LOC_DEVICE, dd = dst->desc.loc == WIND_LOC_DEVICE;
@@ -699,8 +718,7 @@ wind_status route(const wind_kv_pool* src, const wind_kv_pool* dst, int* exec, i
     *path = WIND_PATH_HOST;
     return WIND_OK;
   }
-  const bool same_gpu = memcmp(src->uuid, dst->uuid, 16) == 0;
-  *path = same_gpu ? WIND_PATH_INTRA : WIND_PATH_PEER;
+  *path = local_pair(src, dst) ? WIND_PATH_INTRA : WIND_PATH_PEER;
   if (src->imported && dst->imported)
     return fail(WIND_ERR_UNSUPPORTED, "at least one pool must be local to this process");
   // a local pool on another device of this process: enable peer access from the executing one
@@ -1159,9 +1177,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     q.host_flags = d->desc.loc == WIND_LOC_HOST;
     // GPU-scope publication only when both pools live on the executing GPU (same physical
     // device: every reader of the data and of the flags goes through this GPU's L2)
-    q.sys_scope = force_sys_scope() ||
-                  !(src->desc.loc == WIND_LOC_DEVICE && d->desc.loc == WIND_LOC_DEVICE &&
-                    memcmp(src->uuid, d->uuid, 16) == 0);
+    q.sys_scope = force_sys_scope() || !local_pair(src, d);
     p.sys_scope |= q.sys_scope;
     const int64_t u = p.parts > 1 ? static_cast<int64_t>(it.n) * p.parts
                                   : (static_cast<int64_t>(it.n) + p.group - 1) / p.group;
@@ -1300,9 +1316,7 @@ extern "C" wind_status wind_kv_route(const wind_kv_pool* src, const wind_kv_pool
   // the publication scope run_op chooses: GPU scope only when both pools are device pools on
   // the executing GPU
   if (sys_scope)
-    *sys_scope = force_sys_scope() ||
-                 !(src->desc.loc == WIND_LOC_DEVICE && dst->desc.loc == WIND_LOC_DEVICE &&
-                   memcmp(src->uuid, dst->uuid, 16) == 0);
+    *sys_scope = force_sys_scope() || !local_pair(src, dst);
   return WIND_OK;
 }
 

@@ -20,10 +20,10 @@ timeout -s KILL 1500 ncu --set full --clock-control none --import-source on --re
 echo "full rc=$?" >> $O/${T}_bench.err
 # the N>1 path (pairs over CUDA IPC, all-to-all batch pushes) with every rank on this GPU:
 # a functional check only, NOT multi-GPU bandwidth
-export WIND_BENCH_ONE_DEVICE=1
+export WIND_BENCH_ONE_DEVICE=1 WIND_KV_FORCE_PEER_ROUTE=1
 timeout -s KILL 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 \
   --master-port 29533 bench.py --gpus 2 --steps 5 --warmup 3 --a2a-scale 0.125 --config C1 \
   > $O/${T}_multirank2.log 2>&1; echo "multirank2 rc=$?" >> $O/${T}_multirank2.log
-unset WIND_BENCH_ONE_DEVICE
+unset WIND_BENCH_ONE_DEVICE WIND_KV_FORCE_PEER_ROUTE
 bash scripts/sanitize.sh > $O/${T}_sanitize_summary.txt 2>&1
 ls -la $O > $O/${T}_ls.txt

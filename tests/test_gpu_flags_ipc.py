@@ -156,6 +156,12 @@ def test_ipc_push_and_pull_between_processes():
         remote = wk.Pool.import_(handle, 0)
         assert remote.desc.n_blocks == 90 and remote.nbytes == sh.n_layers * 2 * 90 * sh.chunk_bytes
         src = pattern_pool(sh, 120, 9, 1)
+        # same GPU: INTRA route, unless WIND_KV_FORCE_PEER_ROUTE=1 (test_gpu_sys_scope.py) makes
+        # ops with an imported pool take the PEER route (PEER tuning, system-scope flags)
+        forced = os.environ.get("WIND_KV_FORCE_PEER_ROUTE") == "1"
+        want_path = wk.PATH_PEER if forced else wk.PATH_INTRA
+        assert wk.route(src, remote) == (0, want_path, forced)
+        assert wk.route(remote, src) == (0, want_path, forced)
         rng = np.random.default_rng(4)
         sbt = rng.permutation(120)[:50].astype(np.int32)
         dbt = rng.permutation(90)[:50].astype(np.int32)

@@ -1,4 +1,4 @@
-"""The peer (NVLink) publication path on one GPU.  A peer destination's layer flags are
+"""The peer (NVLink) publication path and peer route on one GPU.  A peer destination's layer flags are
 published at SYSTEM scope (fence.acq_rel.sys, red.relaxed.sys on device-memory flags:
 wind_kv_kernels.cu arrive_layer / bump_flag) — code that only a cross-device op selects,
 and no gpurun call so far had two GPUs.  WIND_KV_FORCE_SYS_SCOPE=1 makes every op publish
@@ -43,3 +43,18 @@ def test_forced_scope_is_reported_by_route():
     r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=env, capture_output=True, text=True,
                        timeout=300)
     assert r.returncode == 0 and "ok" in r.stdout, (r.stdout + r.stderr)[-2000:]
+
+
+def test_forced_peer_route_between_processes():
+    """WIND_KV_FORCE_PEER_ROUTE=1: ops between this process's pool and a pool imported from
+    another process on the same GPU take the PEER route (the PEER tuning — SIMT by default —
+    and system-scope publication): the cross-process push / pull / batched push test and the
+    N = 2 bench path run through it, byte-exact against the oracle."""
+    env = dict(os.environ, WIND_KV_FORCE_PEER_ROUTE="1")
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "-m", "gpu", "-p", "no:cacheprovider",
+                        "tests/test_gpu_flags_ipc.py::test_ipc_push_and_pull_between_processes",
+                        "tests/test_gpu_bench.py::test_bench_multirank_on_one_gpu"],
+                       cwd=ROOT, env=env, capture_output=True, text=True, timeout=1500)
+    tail = (r.stdout + r.stderr)[-3000:]
+    assert r.returncode == 0, tail
+    assert " passed" in r.stdout, tail
