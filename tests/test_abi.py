@@ -145,3 +145,13 @@ def test_plan_compact_worked_example():
     for c in g["cases"]:
         s, d = wk.plan_compact(np.asarray(c["live"], np.uint8))
         assert s.tolist() == c["src_bt"] and d.tolist() == c["dst_bt"], c
+
+
+def test_plan_rebalance_worked_examples():
+    """The library's rebalance planner on the hand-worked R26 examples (tests/golden/)."""
+    import json
+    import os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "r26_rebalance_worked_examples.json")))
+    for c in g["cases"]:
+        out, n = wk.plan_rebalance(c["n_gpus"], c["req_gpu"], c["req_blocks"])
+        assert out.tolist() == c["out_gpu"] and n == c["n_moves"], c

@@ -490,3 +490,14 @@ def test_o6_pairing_worked_example():
         s, d = O.plan_compact(live)
         assert s.tolist() == c["src_bt"] and d.tolist() == c["dst_bt"], c
         assert c["src_bt"] == c["movers"] and c["dst_bt"] == c["holes"]
+
+
+def test_o7_rebalance_worked_examples():
+    """The rebalance rule as read (R26) on hand-worked examples
+    (tests/golden/r26_rebalance_worked_examples.json): pins the CHOICE of moves — which
+    request goes where — not only the plan's invariants."""
+    import json, os
+    g = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "r26_rebalance_worked_examples.json")))
+    for c in g["cases"]:
+        out, n = O.plan_rebalance(c["n_gpus"], c["req_gpu"], c["req_blocks"])
+        assert out.tolist() == c["out_gpu"] and n == c["n_moves"], c
