@@ -76,7 +76,7 @@ def test_plan_compact_large_random():
 
 
 def test_plan_rebalance_matches_oracle():
-    """The plan's CHOICE is parity-unpinned against the paper (a heuristic), but library
+    """The plan's CHOICE follows a reading (R26, a heuristic the paper does not define), but library
     and oracle implement the same stated rule and must agree exactly."""
     from windgen import skewed_placement, lengths_longtail, blocks_for_tokens
     for G in (1, 2, 4, 8):

@@ -339,7 +339,7 @@ def test_compact_preserves_requests():
 # ---------------------------------------------------------------- P7 rebalance plan
 
 def test_plan_rebalance_invariants():
-    """P7 (invariants only; the choice is parity-unpinned): block conservation; at stop,
+    """P7 invariants (the choice is pinned separately, test_o7_rebalance_worked_examples): block conservation; at stop,
     either max load <= target or no request on the most-loaded GPU fits on the least
     loaded one under target; moves only go from above-target to at-most-target GPUs."""
     from windgen import skewed_placement, lengths_longtail, blocks_for_tokens
