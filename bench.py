@@ -70,6 +70,11 @@ class ClockSampler:
                  "-i", str(self.device)], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self._t = threading.Thread(target=self._read, daemon=True)
             self._t.start()
+            # nvidia-smi takes ~0.5-1 s to start: wait for its first sample, so the timed
+            # region that follows is sampled from its start (bounded wait)
+            t_end = time.time() + 5.0
+            while not self.lines and time.time() < t_end and self.proc.poll() is None:
+                time.sleep(0.01)
         except Exception:
             self.proc = None
         return self
@@ -1284,7 +1289,16 @@ def run_gpu(args) -> None:
     launches0 = wk.launch_count()
     step_ms: list = []
     with ClockSampler(local) as clk:
+        t_timed0 = time.time()
         ms_total = time_device(step, args.steps, args.warmup, stream, barrier, per_step=step_ms)
+        t_timed1 = time.time()
+        time.sleep(0.06)  # the sample covering the region's last 50 ms
+    # the samples that arrived during the timed region (all samples if that window is too
+    # short to hold three of them)
+    clk_timed = clk.summary(t_timed0, t_timed1 + 0.06)
+    if clk_timed["samples"] < 3:
+        clk_timed = clk.summary()
+    clk_timed["window_s"] = round(t_timed1 - t_timed0, 3)
     launches = wk.launch_count() - launches0 - (args.warmup if executes() else 0)
     if world > 1:  # every rank's library launches in the timed region (pull: the decode ranks')
         t_l = torch.tensor([float(launches)], dtype=torch.float64)
@@ -1390,7 +1404,7 @@ def run_gpu(args) -> None:
             "step_ms_rank0": {"p10": round(float(np.percentile(step_ms, 10)), 4),
                               "p50": round(float(np.percentile(step_ms, 50)), 4),
                               "p90": round(float(np.percentile(step_ms, 90)), 4)},
-            "clocks": clk.summary(),
+            "clocks": clk_timed,
             # the paper's only migration number, as context (A800, not a target): one
             # 2048-token OPT-13B request = 1.5625 GiB, "~65 ms" over PCIe Gen4 x16
             "paper_context": {
