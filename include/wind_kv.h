@@ -278,7 +278,11 @@ wind_status wind_kv_layer_ticket(const wind_kv_pool* dst, uint32_t* ticket);
 /* Makes `consumer` wait (device-side, no host sync) until dst's layer_done for global
  * `layer` reaches `ticket` (wrap-safe >=), i.e. until that many ops have landed that
  * layer.  Uses cuStreamWaitValue32(GEQ) on the flag, local to dst.  When ops into one
- * pool are issued on one stream, flag >= t means ops 1..t are complete for that layer. */
+ * pool are issued on one stream, flag >= t means ops 1..t are complete for that layer.
+ * Under CUDA graph capture the ticket is a constant of the graph: every replay waits for
+ * the capture-time count, which the first replay's ops already reach — so a graph that
+ * contains both the ops and their waits orders them correctly on its first replay only;
+ * for repeated replays, wait outside the graph (or re-capture). */
 wind_status wind_kv_layer_wait(const wind_kv_pool* dst, int32_t layer, uint32_t ticket,
                                void* consumer);
 

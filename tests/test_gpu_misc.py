@@ -176,3 +176,55 @@ def test_many_concurrent_ops_across_streams():
         np.testing.assert_array_equal(p.tensor().cpu().numpy(), want)
         assert [p.layer_count(l) for l in range(L)] == [1] * L
     assert one.layer_ticket() == 40 and [one.layer_count(l) for l in range(L)] == [40] * L
+
+
+def test_ops_enqueued_from_many_host_threads():
+    """Four host threads enqueue 40 ops each at the same time (ctypes releases the GIL inside
+    the library), each thread into its own destination pools on its own stream, from one
+    shared source pool: every destination byte-exact vs the oracle, every ticket and flag
+    right (the per-device counter ring, the pools' ticket counters and the tuning table are
+    shared state)."""
+    import threading
+    import oracle as O
+    L, H, d, bs, eb = 4, 2, 64, 16, 2
+    rng = np.random.default_rng(11)
+    src = wk.Pool(L, H, d, bs, eb, 64)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    plans = []
+    for t in range(4):
+        pools = [wk.Pool(L, H, d, bs, eb, 24) for _ in range(4)]
+        for p in pools:
+            p.tensor().zero_()
+        ops = []
+        for k in range(40):
+            sbt = rng.permutation(64)[:12].astype(np.int32)
+            dbt = rng.permutation(24)[:12].astype(np.int32)
+            lo = int(rng.integers(0, L))
+            ops.append((k % 4, torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV),
+                        sbt, dbt, lo, lo + 1))
+        plans.append((pools, torch.cuda.Stream(DEV), ops))
+    torch.cuda.synchronize()
+    errors = []
+
+    def worker(pools, stream, ops):
+        try:
+            for j, ts, td, _, _, lo, hi in ops:
+                wk.migrate(src, ts, pools[j], td, layer_lo=lo, layer_hi=hi, stream=stream)
+        except Exception as e:  # noqa: BLE001 — reported below
+            errors.append(e)
+    threads = [threading.Thread(target=worker, args=pl) for pl in plans]
+    for th in threads:
+        th.start()
+    for th in threads:
+        th.join()
+    torch.cuda.synchronize()
+    assert not errors, errors
+    g = lambda nb: O.Geom(0, L, H, d, bs, eb, nb)  # noqa: E731
+    for pools, _, ops in plans:
+        want = [np.zeros(p.nbytes, np.uint8) for p in pools]
+        for j, _, _, sbt, dbt, lo, hi in ops:  # one stream per thread: in order
+            assert O.migrate(s0, g(64), sbt, want[j], g(24), dbt, lo, hi) == O.OK
+        for p, w in zip(pools, want):
+            np.testing.assert_array_equal(p.tensor().cpu().numpy(), w)
+            assert p.layer_ticket() == 10 and [p.layer_count(l) for l in range(L)] == [10] * L
