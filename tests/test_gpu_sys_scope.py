@@ -3,8 +3,8 @@ published at SYSTEM scope (fence.acq_rel.sys, red.relaxed.sys on device-memory f
 wind_kv_kernels.cu arrive_layer / bump_flag) — code that only a cross-device op selects,
 and no gpurun call so far had two GPUs.  WIND_KV_FORCE_SYS_SCOPE=1 makes every op publish
 that way, so the flag-ordering property test, the layer-streamed prefill hand-off, the
-one-launch all-to-all and whole-pool parity run here through the system-scope code with
-the data on one device.  Run in a subprocess: the variable is read once per process."""
+one-launch all-to-all, whole-pool parity and the 400-case random fuzz run here through the
+system-scope code with the data on one device.  Run in a subprocess: the variable is read once per process."""
 import os
 import subprocess
 import sys
@@ -21,6 +21,7 @@ NODES = [
     "tests/test_gpu_parity.py::test_migrate_c1_all_kernels",
     "tests/test_gpu_parity.py::test_run_coalescing_across_warp_windows",
     "tests/test_gpu_heads.py",
+    "tests/test_gpu_fuzz.py",  # 400 random ops (geometry, tables, windows, kernels, swaps)
 ]
 
 
