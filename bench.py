@@ -334,8 +334,11 @@ def run_scenarios(wk, device, peaks, steps=10, warmup=3) -> dict:
     del dpool, dpool2, hpool, hbuf, dbuf
     torch.cuda.empty_cache()
 
-    # (5) interference with a co-running decode stream (C3)
+    # (5) interference with a co-running decode stream (C3): decode attention alone (the
+    #     worst case: every byte of the step is KV), then a whole decode step (GEMMs too)
     out["c3_interference"] = run_interference(wk, device, peaks)
+    torch.cuda.empty_cache()
+    out["c3_interference_decode_step"] = run_interference(wk, device, peaks, victim_kind="decode_step")
     torch.cuda.empty_cache()
 
     # (6) stall-free rescheduling of P:120's request (NEXT-1)
@@ -796,7 +799,7 @@ def run_stall_free(wk, device, cap_ctas: int = 16) -> dict:
                 "pause_ms": round(resb.pause_ms, 3), "blocks_sent": resb.blocks_sent}}
 
 
-def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict:
+def run_interference(wk, device, peaks, n_victim_steps=50, configs=None, victim_kind="attention") -> dict:
     """S§8(d) interference, C3 (OPT-66B KV, 64 layers x 72 heads x d 128, fp16): the victim
     is paged decode attention over 16 x 2048 resident tokens (the Fig. 8 decode set,
     P:251) = 72 GiB of KV read per step (64 layer launches) on a HIGH-priority stream; the
@@ -804,15 +807,25 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     side stream, looped to cover every victim step.  On one GPU the migration is
     intra-device (reads AND writes this HBM); a CTA cap emulates the source-side HBM load
     of an NVLink push (8 CTAs ~ 365 GB/s payload = 730 GB/s of DRAM traffic, about what a
-    770 GB/s peer push reads on its source GPU)."""
+    770 GB/s peer push reads on its source GPU).
+
+    victim_kind="decode_step": a victim closer to a whole decode step of OPT-66B on one
+    TP-2 rank (Table 3 placements are TP-2): per layer the QKV projection, paged
+    attention over this rank's 36 heads of the 16 x 2048-token set, the output projection
+    and the MLP — fp16 GEMMs (cuBLAS, harness only) against one layer's weight shard
+    (1.02 GB, re-read every layer: it cannot stay in the 126 MB L2) — so a step streams
+    65 GB of weights plus 36 GiB of KV."""
     import torch
     import victim
-    from windgen import migration_case, SHAPES
+    from windgen import migration_case, SHAPES, KVShape
     sh = SHAPES["C3"]
     dev = torch.device("cuda", device)
     B, ctx_len, bs = 16, 2048, sh.block_size
     nbv = B * ctx_len // bs
-    vpool = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, bs, sh.elem_bytes, nbv, device=device)
+    full_step = victim_kind == "decode_step"
+    vsh = KVShape("OPT-66B TP-2 shard", sh.n_layers, sh.n_kv_heads // 2, sh.head_dim, sh.elem_bytes) \
+        if full_step else sh
+    vpool = wk.Pool(vsh.n_layers, vsh.n_kv_heads, vsh.head_dim, bs, vsh.elem_bytes, nbv, device=device)
     vt = vpool.tensor().view(torch.float16)
     g = torch.Generator(device=dev).manual_seed(0)
     step_elems = 1 << 28
@@ -822,19 +835,41 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     perm = torch.randperm(nbv, generator=torch.Generator().manual_seed(1)).to(torch.int32)
     bt = perm.view(B, ctx_len // bs).to(dev)
     ctx = torch.full((B,), ctx_len, dtype=torch.int32, device=dev)
-    q = torch.randn(B, sh.n_kv_heads, sh.head_dim, device=dev, dtype=torch.float16)
+    hv = vsh.n_kv_heads
+    q = torch.randn(B, hv, sh.head_dim, device=dev, dtype=torch.float16)
     bps = 64  # sweep r01: 0.978 of HBM on this shape
-    scratch = torch.empty(victim.scratch_floats(B, sh.n_kv_heads, ctx_len // bs, bps), device=dev)
-    out = torch.empty(B, sh.n_kv_heads, sh.head_dim, device=dev)
-    plane = nbv * sh.chunk_bytes
+    scratch = torch.empty(victim.scratch_floats(B, hv, ctx_len // bs, bps), device=dev)
+    out = torch.empty(B, hv, sh.head_dim, device=dev)
+    plane = nbv * vsh.chunk_bytes
     hi_s = torch.cuda.Stream(device, priority=-1)
     lo_s = torch.cuda.Stream(device, priority=0)
+    if full_step:  # one TP-2 layer's weight shard, fp16, re-read by every layer
+        Hd, Hs = 9216, hv * sh.head_dim  # hidden size of OPT-66B, this rank's attention width
+        gw = torch.Generator(device=dev).manual_seed(2)
+        w_qkv = torch.randn(Hd, 3 * Hs, device=dev, dtype=torch.float16, generator=gw) * 0.01
+        w_o = torch.randn(Hs, Hd, device=dev, dtype=torch.float16, generator=gw) * 0.01
+        w_1 = torch.randn(Hd, 2 * Hd, device=dev, dtype=torch.float16, generator=gw) * 0.01
+        w_2 = torch.randn(2 * Hd, Hd, device=dev, dtype=torch.float16, generator=gw) * 0.01
+        h0 = torch.randn(B, Hd, device=dev, dtype=torch.float16, generator=gw)
+        w_bytes = sum(w.numel() * 2 for w in (w_qkv, w_o, w_1, w_2))
 
     def victim_step_on(st):
-        for l in range(sh.n_layers):
-            kp = vpool.base + (2 * l) * plane
-            victim.decode_attention(q, kp, kp + plane, bt, ctx, sh.n_kv_heads, bs, scratch, out,
-                                    blocks_per_split=bps, stream=st.cuda_stream)
+        if not full_step:
+            for l in range(sh.n_layers):
+                kp = vpool.base + (2 * l) * plane
+                victim.decode_attention(q, kp, kp + plane, bt, ctx, hv, bs, scratch, out,
+                                        blocks_per_split=bps, stream=st.cuda_stream)
+            return
+        with torch.cuda.stream(st):
+            h = h0
+            for l in range(sh.n_layers):
+                qkv = h @ w_qkv
+                ql = qkv[:, :Hs].contiguous().view(B, hv, sh.head_dim)
+                kp = vpool.base + (2 * l) * plane
+                victim.decode_attention(ql, kp, kp + plane, bt, ctx, hv, bs, scratch, out,
+                                        blocks_per_split=bps, stream=st.cuda_stream)
+                h1 = h + out.view(B, Hs).half() @ w_o
+                h = torch.tanh(h1 + torch.nn.functional.gelu(h1 @ w_1) @ w_2)
 
     def victim_step():
         victim_step_on(hi_s)
@@ -862,10 +897,14 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     torch.cuda.synchronize()
     alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]
     t_alone = float(np.median(alone))
-    kv_read = B * ctx_len * sh.n_layers * 2 * sh.n_kv_heads * sh.head_dim * sh.elem_bytes
+    kv_read = B * ctx_len * sh.n_layers * 2 * hv * sh.head_dim * sh.elem_bytes
+    step_bytes = kv_read + (w_bytes * sh.n_layers if full_step else 0)
     res = {"victim_ms_alone": round(t_alone, 3),
-           "victim_hbm_frac": round(kv_read / t_alone / 1e6 / peaks["hbm_gbs"], 3),
-           "victim": "paged decode attention, 16 x 2048 tok, 64 layers, 72 heads (C3)"}
+           "victim_hbm_frac": round(step_bytes / t_alone / 1e6 / peaks["hbm_gbs"], 3),
+           "victim": ("OPT-66B decode step on one TP-2 rank: QKV, paged attention (36 heads, "
+                      "16 x 2048 tok), output projection, MLP; 64 layers; weights "
+                      f"{w_bytes * sh.n_layers / 1e9:.1f} GB + KV {kv_read / 1e9:.1f} GB per step"
+                      if full_step else "paged decode attention, 16 x 2048 tok, 64 layers, 72 heads (C3)")}
 
     case = migration_case("C3")
     src = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
@@ -885,6 +924,14 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None) -> dict
     # purpose (the bytes are never read; release builds do not check table content)
     sink = wk.Pool(sh.n_layers, sh.n_kv_heads, sh.head_dim, sh.block_size, sh.elem_bytes, 1, device=device)
     zeros_t = torch.zeros(case.n, dtype=torch.int32, device=dev)
+    if configs is None and full_step:  # the whole-decode-step victim: the informative rows
+        configs = ([("control_no_migration", {**saved, "null_feeder": True}),
+                    ("cap2", {**saved, "max_ctas": 2})] +
+                   [(f"rate{r}GBs", {**saved, "max_ctas": 0, "rate_mbps": r * 1000}) for r in (50, 150)] +
+                   [("copy_engines_rate50GBs", {**saved, "kernel": wk.KERNEL_COPY_ENGINE, "rate_mbps": 50000}),
+                    ("swap_out_sm_default", {"op": "swap_out", **saved_host, "kernel": wk.KERNEL_TMA}),
+                    ("push_source_proxy_rate700GBs", {**saved, "op": "push_source_proxy", "max_ctas": 0,
+                                                      "rate_mbps": 700000})])
     configs = configs or (
         [("control_no_migration", {**saved, "null_feeder": True})] +
         [(f"cap{c or 'none'}", {**saved, "max_ctas": c}) for c in (2, 4, 8, 16, 0)] +

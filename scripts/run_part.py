@@ -1,5 +1,5 @@
 """Development helper: one bench.py scenario alone, printed as one JSON line.
-usage: python scripts/run_part.py c1_intra|interference|burst|proxy|handoff|stall_free|pressure|next3|policy"""
+usage: python scripts/run_part.py c1_intra|interference|decode_step|burst|proxy|handoff|stall_free|pressure|next3|policy"""
 import json
 import os
 import sys
@@ -12,6 +12,7 @@ peaks = bench.load_peaks()
 name = sys.argv[1]
 fn = {"c1_intra": lambda: bench.run_c1_intra(wk, 0, peaks),
       "interference": lambda: bench.run_interference(wk, 0, peaks),
+      "decode_step": lambda: bench.run_interference(wk, 0, peaks, victim_kind="decode_step"),
       # trickle rows only (then the burst rows, which run_interference always adds)
       "burst": lambda: bench.run_interference(wk, 0, peaks, configs=[
           (f"rate{r}GBs", {**wk.get_tuning(wk.PATH_INTRA), "max_ctas": 0, "rate_mbps": r * 1000})
