@@ -1,5 +1,5 @@
 """Development helper: one bench.py scenario alone, printed as one JSON line.
-usage: python scripts/run_part.py c1_intra|interference|decode_step|burst|proxy|handoff|stall_free|pressure|next3|policy"""
+usage: python scripts/run_part.py c1_intra|interference|decode_step|pacer_footprint|burst|proxy|handoff|stall_free|pressure|next3|policy"""
 import json
 import os
 import sys
@@ -13,6 +13,15 @@ name = sys.argv[1]
 fn = {"c1_intra": lambda: bench.run_c1_intra(wk, 0, peaks),
       "interference": lambda: bench.run_interference(wk, 0, peaks),
       "decode_step": lambda: bench.run_interference(wk, 0, peaks, victim_kind="decode_step"),
+      # rate-limited kernels with a smaller on-SM footprint, next to the decode-step victim
+      "pacer_footprint": lambda: bench.run_interference(wk, 0, peaks, victim_kind="decode_step", configs=[
+          (name, {**wk.get_tuning(wk.PATH_INTRA), "max_ctas": 0, "rate_mbps": 150000, **kw})
+          for name, kw in (("rate150_tma_48kx4", {}),
+                           ("rate150_tma_16kx4", {"stage_bytes": 16384, "stages": 4, "store_lag": 2}),
+                           ("rate150_tma_8kx4", {"stage_bytes": 8192, "stages": 4, "store_lag": 2}),
+                           ("rate150_simt", {"kernel": wk.KERNEL_SIMT, "stage_bytes": 32768}),
+                           ("rate50_simt", {"kernel": wk.KERNEL_SIMT, "stage_bytes": 32768,
+                                            "rate_mbps": 50000}))]),
       # trickle rows only (then the burst rows, which run_interference always adds)
       "burst": lambda: bench.run_interference(wk, 0, peaks, configs=[
           (f"rate{r}GBs", {**wk.get_tuning(wk.PATH_INTRA), "max_ctas": 0, "rate_mbps": r * 1000})
