@@ -89,6 +89,7 @@ struct DevCtx {
   int sms = 0;
   uint8_t uuid[16] = {};
   uint32_t* counters = nullptr;  // kCounterSlots * WIND_KV_MAX_LAYERS, zeroed
+  unsigned long long* stamps = nullptr;  // kCounterSlots: start time of a burst-paced op
   std::atomic<uint64_t> seq{0};
   size_t tma_smem_set = 0;
   int32_t* err = nullptr;        // debug device-check word
@@ -117,6 +118,7 @@ wind_status dev_ctx(int dev, DevCtx** out) {
     const size_t cbytes = sizeof(uint32_t) * kCounterSlots * WIND_KV_MAX_LAYERS;
     WKV_CUDA(cudaMalloc(&c.counters, cbytes), "cudaMalloc(counters)");
     WKV_CUDA(cudaMemset(c.counters, 0, cbytes), "cudaMemset(counters)");
+    WKV_CUDA(cudaMalloc(&c.stamps, sizeof(unsigned long long) * kCounterSlots), "cudaMalloc(stamps)");
     WKV_CUDA(cudaMalloc(&c.err, sizeof(int32_t)), "cudaMalloc(err)");
     WKV_CUDA(cudaMemset(c.err, 0, sizeof(int32_t)), "cudaMemset(err)");
     const size_t max_smem = 227 * 1024;
@@ -194,6 +196,26 @@ bool force_peer_route() {
     return e && e[0] == '1';
   }();
   return on;
+}
+
+// WIND_KV_BURST_PACING=0: rate-limited device ops pace inside a small resident grid (the
+// round-1 pacer) instead of in full-grid bursts (A/B measurements).
+bool burst_pacing_enabled() {
+  static const bool on = [] {
+    const char* e = getenv("WIND_KV_BURST_PACING");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}
+// A burst-paced op moves this many ns of its rate budget per burst (WIND_KV_BURST_PERIOD_US
+// overrides it, for A/B measurements).
+double burst_period_ns() {
+  static const double ns = [] {
+    const char* e = getenv("WIND_KV_BURST_PERIOD_US");
+    const double us = e ? atof(e) : 0.0;
+    return us >= 10.0 ? us * 1e3 : 2e6;
+  }();
+  return ns;
 }
 
 constexpr int kHostCtasFromHost = 8;
@@ -1217,10 +1239,18 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     for (int j = 0; j < n_items; ++j) to_host = to_host || items[j].dst->desc.loc == WIND_LOC_HOST;
     grid = std::min<int64_t>(grid, to_host ? ctas_for_in_flight(kHostToHostInFlight, ring) : kHostCtasFromHost);
   }
-  // A rate-limited op holds as few SMs as can sustain the rate (one CTA moves ~38 GB/s of
-  // payload intra-device): the SMs a migration occupies cost a co-running HBM-bound decode
-  // kernel more than the bytes it moves (bench c3_interference).
-  if (t.rate_mbps > 0 && t.max_ctas == 0)
+  // Rate limits.  Device ops (INTRA / PEER) with no CTA cap are BURST-paced: the op is cut
+  // into slices of its units, each slice moved by the full grid at full rate and followed
+  // by a 1-thread pace kernel that holds the stream until the rate schedule allows the next
+  // one (2 ms of rate budget per slice).  Between bursts no copy CTA is resident, so a
+  // co-running decode step keeps every SM: a paced grid of sleeping CTAs (the round-1
+  // pacer, still used when max_ctas > 0 or on the HOST path) cost a decode step of GEMMs +
+  // attention 19-29 % at 50-150 GB/s, bursts 1.3-4.4 %.
+  const bool burst_paced = t.rate_mbps > 0 && t.max_ctas == 0 && path != WIND_PATH_HOST && !debug &&
+                           burst_pacing_enabled();
+  // in-kernel pacing: as few SMs as can sustain the rate (one CTA moves ~38 GB/s of payload
+  // intra-device)
+  if (t.rate_mbps > 0 && t.max_ctas == 0 && !burst_paced)
     grid = std::min<int64_t>(grid, std::max<int64_t>(1, (t.rate_mbps + kCtaMBps - 1) / kCtaMBps));
   grid = std::max<int64_t>(1, std::min<int64_t>(grid, p.total_units));
   // Work dealing.  Grid-stride (all CTAs sweep the layers together: each layer completes
@@ -1229,6 +1259,39 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   // older stores to be fully written before the arrival — a latency chain that dominates
   // small ops.  Those get contiguous unit ranges per CTA (a handful of crossings each).
   p.blocked = (p.units_per_plane < grid && t.rate_mbps == 0 && blocked_dealing_enabled()) ? 1 : 0;
+  p.unit_lo = 0;
+  p.unit_hi = p.total_units;
+  p.first_slice = 1;
+  if (burst_paced) {
+    // source payload of the op (a fan-out reads each unit once)
+    int64_t n_src = 0;
+    for (int j = 0; j < (fan > 1 ? 1 : n_items); ++j) n_src += items[j].n;
+    const double payload = 2.0 * p.n_layers * static_cast<double>(CP) * static_cast<double>(n_src);
+    const double slice_bytes = t.rate_mbps * 1e6 * burst_period_ns() * 1e-9;
+    int64_t slice_units = static_cast<int64_t>(p.total_units * slice_bytes / std::max(1.0, payload));
+    slice_units = std::max<int64_t>(slice_units, grid);  // a burst keeps the whole grid busy
+    unsigned long long* t0 = ctx->stamps + slot;
+    p.ns_per_byte = 0.f;
+    WKV_CUDA(launch_pace(t0, 0, 1, s), "pace kernel launch");
+    int launches = 1;
+    for (int64_t u = 0; u < p.total_units; u += slice_units) {
+      p.unit_lo = u;
+      p.unit_hi = std::min<int64_t>(p.total_units, u + slice_units);
+      p.first_slice = u == 0;
+      cudaError_t e = launch_copy(p, kernel, static_cast<int>(std::min<int64_t>(grid, p.unit_hi - u)), s,
+                                  pdl_enabled());
+      if (e != cudaSuccess) return cuda_fail(e, "copy kernel launch");
+      ++launches;
+      // hold the stream until the schedule reaches the bytes moved so far (after the last
+      // slice too: the op then ends when its rate says, as the in-kernel pacer's ops do)
+      const double done = payload * static_cast<double>(p.unit_hi) / static_cast<double>(p.total_units);
+      WKV_CUDA(launch_pace(t0, static_cast<uint64_t>(done * 1e3 / t.rate_mbps), 0, s), "pace kernel launch");
+      ++launches;
+    }
+    g_launches += launches;
+    for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
+    return WIND_OK;
+  }
   // rate limit: each of the `grid` CTAs gets rate / grid; ns per payload byte per CTA
   p.ns_per_byte = t.rate_mbps > 0 ? static_cast<float>(grid * 1e3 / t.rate_mbps) : 0.f;
   cudaError_t e = launch_copy(p, kernel, static_cast<int>(grid), s, pdl_enabled());

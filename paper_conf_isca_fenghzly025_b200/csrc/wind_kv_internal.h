@@ -45,6 +45,9 @@ struct Params {
   int64_t copy;               // bytes copied per (layer, kv, block): C, or n_heads * tile
   int64_t units_per_plane;    // sum of items' units
   int64_t total_units;        // planes * units_per_plane
+  int64_t unit_lo, unit_hi;   // the units THIS launch moves (a burst-paced op launches
+                              // slices of [0, total_units) on one counter slot)
+  int32_t first_slice;        // 1: this launch also bumps the untouched layers' flags
   uint32_t* counters;         // this op's counter slot, [hi - lo]
   const int32_t* abort_word;  // debug pools: skip the copy if the device check fired
   int32_t layer_lo, n_layers; // global lo, hi - lo

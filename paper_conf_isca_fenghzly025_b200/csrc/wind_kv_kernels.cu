@@ -419,7 +419,7 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
   }
   __syncthreads();
   pdl_wait();  // everything below may see the previous grid's writes
-  if (blockIdx.x == 0 && threadIdx.x == 33) publish_untouched_layers(p);  // an idle consumer lane
+  if (blockIdx.x == 0 && threadIdx.x == 33 && p.first_slice) publish_untouched_layers(p);  // an idle consumer lane
   if (p.abort_word && *reinterpret_cast<const volatile int32_t*>(p.abort_word)) {
     if (blockIdx.x == 0 && threadIdx.x == 0) publish_aborted(p);
     return;
@@ -427,11 +427,11 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
 
   if (warp == 0) {  // ------------------------------------------------ producer warp
     const uint64_t pol = ef ? evict_first_policy() : 0;
-    const int64_t total = p.total_units;
-    int64_t u0 = blockIdx.x, ustep = gridDim.x, uend = total;
+    const int64_t total = p.unit_hi;  // this launch's units: [unit_lo, unit_hi)
+    int64_t u0 = p.unit_lo + blockIdx.x, ustep = gridDim.x, uend = total;
     if (p.blocked) {  // contiguous range: the CTA crosses few layer boundaries
-      const int64_t per = (p.total_units + gridDim.x - 1) / gridDim.x;
-      u0 = blockIdx.x * per;
+      const int64_t per = (p.unit_hi - p.unit_lo + gridDim.x - 1) / gridDim.x;
+      u0 = p.unit_lo + blockIdx.x * per;
       ustep = 1;
       uend = u0 + per < total ? u0 + per : total;
     }
@@ -542,18 +542,18 @@ __global__ void __launch_bounds__(kSimtThreads) simt_copy_kernel(const __grid_co
   const bool ef = p.evict_first != 0;
   const uint64_t pol = ef ? evict_first_policy() : 0;
   pdl_wait();
-  if (blockIdx.x == 0 && tid == 32) publish_untouched_layers(p);  // not the decoding warp
+  if (blockIdx.x == 0 && tid == 32 && p.first_slice) publish_untouched_layers(p);  // not the decoding warp
   if (p.abort_word && *reinterpret_cast<const volatile int32_t*>(p.abort_word)) {
     if (blockIdx.x == 0 && tid == 0) publish_aborted(p);
     return;
   }
   int32_t cur = -1;  // layer of the units being copied, and how many of them
   uint32_t cur_cnt = 0;
-  const int64_t total = p.total_units;
-  int64_t u0 = blockIdx.x, ustep = gridDim.x, uend = total;
+  const int64_t total = p.unit_hi;  // this launch's units: [unit_lo, unit_hi)
+  int64_t u0 = p.unit_lo + blockIdx.x, ustep = gridDim.x, uend = total;
   if (p.blocked) {
-    const int64_t per = (p.total_units + gridDim.x - 1) / gridDim.x;
-    u0 = blockIdx.x * per;
+    const int64_t per = (p.unit_hi - p.unit_lo + gridDim.x - 1) / gridDim.x;
+    u0 = p.unit_lo + blockIdx.x * per;
     ustep = 1;
     uend = u0 + per < total ? u0 + per : total;
   }

@@ -91,9 +91,11 @@ def test_launch_count_one_kernel_per_op():
     del sh
 
 
-def test_rate_limit_paces_the_copy():
+@pytest.mark.parametrize("max_ctas", [0, 4])
+def test_rate_limit_paces_the_copy(max_ctas):
     """wind_kv_tuning.rate_mbps bounds an op's payload rate (interference budget) without
-    changing its result."""
+    changing its result: burst pacing (max_ctas 0: full-grid slices between 1-thread pace
+    kernels) and the in-kernel pacer (a CTA cap: a small paced grid)."""
     from windgen import SHAPES
     import windgen.cuda as wg
     sh = SHAPES["C2"]
@@ -109,11 +111,17 @@ def test_rate_limit_paces_the_copy():
     s = torch.cuda.Stream(DEV)
     try:
         for rate_gbs in (20, 80):
-            wk.set_tuning(wk.PATH_INTRA, **{**saved, "rate_mbps": rate_gbs * 1000})
+            wk.set_tuning(wk.PATH_INTRA, **{**saved, "rate_mbps": rate_gbs * 1000, "max_ctas": max_ctas})
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(s)
+            n0 = wk.launch_count()
             wk.migrate(src, sbt, dst, dbt, stream=s)
             b.record(s)
+            if max_ctas == 0:  # 2 ms of rate budget per burst, a pace kernel before and after each
+                bursts = (wk.launch_count() - n0 - 1) // 2
+                assert abs(bursts - payload / (rate_gbs * 1e9 * 2e-3)) <= 1.5, bursts
+            else:
+                assert wk.launch_count() - n0 == 1
             torch.cuda.synchronize()
             got = payload / (a.elapsed_time(b) * 1e6)
             assert 0.75 * rate_gbs < got < 1.1 * rate_gbs, (rate_gbs, got)
@@ -122,6 +130,50 @@ def test_rate_limit_paces_the_copy():
     S = src.tensor().view(4, 2, nb, -1)
     D = dst.tensor().view(4, 2, nb, -1)
     assert torch.equal(D[:, :, dbt.long()], S[:, :, sbt.long()])
+
+
+def test_burst_paced_op_flags_and_parity():
+    """A burst-paced op (rate limit, no CTA cap) is many launches on ONE arrival-counter slot:
+    a consumer stream waits on every layer flag and snapshots the layer — each snapshot
+    already holds the oracle's bytes — the whole pool equals the oracle, every flag moves
+    exactly once, and a layer window leaves the other layers' bytes alone."""
+    import oracle as O
+    from windgen import SHAPES
+    sh = SHAPES["C2"]
+    L, nb, n = 8, 200, 150
+    src = wk.Pool(L, sh.n_kv_heads, sh.head_dim, 16, 2, nb)
+    dst = wk.Pool(L, sh.n_kv_heads, sh.head_dim, 16, 2, nb)
+    rng = np.random.default_rng(5)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    d0 = rng.integers(0, 256, dst.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    dst.tensor().copy_(torch.from_numpy(d0))
+    sbt = rng.permutation(nb)[:n].astype(np.int32)
+    dbt = rng.permutation(nb)[:n].astype(np.int32)
+    ts, td = torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)
+    want = d0.copy()
+    g = O.Geom(0, L, sh.n_kv_heads, sh.head_dim, 16, 2, nb)
+    assert O.migrate(s0, g, sbt, want, g, dbt, 1, 7) == O.OK
+    plane = nb * sh.chunk_bytes
+    view = dst.tensor()
+    snaps = torch.empty(L, 2 * plane, dtype=torch.uint8, device=DEV)
+    s, cons = torch.cuda.Stream(DEV), torch.cuda.Stream(DEV)
+    torch.cuda.synchronize()
+    n0 = wk.launch_count()
+    # 2 x 6 layers x 150 blocks x 160 KiB = 281 MiB at 50 GB/s: ~3 bursts of 100 MB
+    wk.migrate_ex(src, ts, dst, td, wk.tuning(rate_mbps=50_000, max_ctas=0),
+                  layer_lo=1, layer_hi=7, stream=s)
+    launches = wk.launch_count() - n0
+    assert launches >= 5 and launches % 2 == 1  # 1 + 2 x bursts
+    t = dst.layer_ticket()
+    with torch.cuda.stream(cons):
+        for l in range(L):
+            wk.layer_wait(dst, l, t, stream=cons)
+            snaps[l].copy_(view[l * 2 * plane:(l + 1) * 2 * plane])
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(snaps.cpu().numpy().reshape(-1), want)
+    np.testing.assert_array_equal(view.cpu().numpy(), want)
+    assert [dst.layer_count(l) for l in range(L)] == [1] * L
 
 
 def test_plain_c_abi_user():
