@@ -358,7 +358,17 @@ typedef struct {
   int32_t store_lag;   /* TMA: stores allowed in flight per CTA (0 = stages / 2) */
   int32_t rate_mbps;   /* payload rate limit of one op in MB/s (0 = unlimited): bounds the
                           HBM / link share a migration takes from co-running decode
-                          (S§8(d) interference); paced per CTA with %globaltimer */
+                          (S§8(d) interference).  INTRA / PEER ops with max_ctas == 0 are
+                          BURST-paced: slices of the op (2 ms of rate budget each) run on
+                          the full grid at full rate, each followed by a 1-thread pace
+                          kernel that holds the stream until the schedule allows the next,
+                          so no copy CTA stays resident between bursts (1 + 2 x slices
+                          launches; flags, tickets and results are one op's).  With
+                          max_ctas > 0, and on the HOST path, the grid's CTAs pace
+                          themselves with %globaltimer (one launch).  Either way the op ends
+                          when its rate schedule says.  For background moves next to a
+                          decode loop, one full-rate op per decode step is cheaper still
+                          (DESIGN.md §6). */
 } wind_kv_tuning;
 
 wind_status wind_kv_set_tuning(int32_t path, const wind_kv_tuning* t);
