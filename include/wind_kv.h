@@ -360,7 +360,7 @@ typedef struct {
                           HBM / link share a migration takes from co-running decode
                           (S§8(d) interference).  INTRA / PEER ops with max_ctas == 0 are
                           BURST-paced: slices of the op (2 ms of rate budget each) run on
-                          the full grid at full rate, each followed by a 1-thread pace
+                          half the grid at full rate, each followed by a 1-thread pace
                           kernel that holds the stream until the schedule allows the next,
                           so no copy CTA stays resident between bursts (1 + 2 x slices
                           launches; flags, tickets and results are one op's).  With

@@ -1269,6 +1269,13 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     const double payload = 2.0 * p.n_layers * static_cast<double>(CP) * static_cast<double>(n_src);
     const double slice_bytes = t.rate_mbps * 1e6 * burst_period_ns() * 1e-9;
     int64_t slice_units = static_cast<int64_t>(p.total_units * slice_bytes / std::max(1.0, payload));
+    // a burst runs on half the grid: nearly the full HBM rate (one CTA moves ~38 GB/s), and
+    // half the SMs stay with the co-running work (sweep, profiles/r02/burst_pacer/: 74 CTAs
+    // beat 148 / 37 / 16 next to both victims); WIND_KV_BURST_CTAS overrides it (A/B)
+    grid = std::max<int64_t>(1, grid / 2);
+    if (const char* e = getenv("WIND_KV_BURST_CTAS"))
+      grid = std::max<int64_t>(1, atoi(e) > 0 ? atoi(e) : grid);
+    grid = std::min<int64_t>(grid, p.total_units);
     slice_units = std::max<int64_t>(slice_units, grid);  // a burst keeps the whole grid busy
     unsigned long long* t0 = ctx->stamps + slot;
     p.ns_per_byte = 0.f;

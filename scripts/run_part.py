@@ -1,5 +1,5 @@
 """Development helper: one bench.py scenario alone, printed as one JSON line.
-usage: python scripts/run_part.py c1_intra|interference|decode_step|pacer_footprint|burst_period|burst|proxy|handoff|stall_free|pressure|next3|policy"""
+usage: python scripts/run_part.py c1_intra|interference|decode_step|pacer_footprint|burst_period|burst_grid|burst|proxy|handoff|stall_free|pressure|next3|policy"""
 import json
 import os
 import sys
@@ -13,6 +13,9 @@ name = sys.argv[1]
 fn = {"c1_intra": lambda: bench.run_c1_intra(wk, 0, peaks),
       "interference": lambda: bench.run_interference(wk, 0, peaks),
       "decode_step": lambda: bench.run_interference(wk, 0, peaks, victim_kind="decode_step"),
+      "burst_grid": lambda: {v: bench.run_interference(wk, 0, peaks, victim_kind=v, configs=[
+          (f"rate{r}GBs", {**wk.get_tuning(wk.PATH_INTRA), "max_ctas": 0, "rate_mbps": r * 1000})
+          for r in (50, 150)]) for v in ("attention", "decode_step")},
       "burst_period": lambda: bench.run_interference(wk, 0, peaks, victim_kind="decode_step", configs=[
           (f"rate{r}GBs", {**wk.get_tuning(wk.PATH_INTRA), "max_ctas": 0, "rate_mbps": r * 1000})
           for r in (50, 150, 300)]),
