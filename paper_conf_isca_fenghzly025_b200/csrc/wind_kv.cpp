@@ -199,7 +199,7 @@ bool force_peer_route() {
 }
 
 // WIND_KV_BURST_PACING=0: rate-limited device ops pace inside a small resident grid (the
-// round-1 pacer) instead of in full-grid bursts (A/B measurements).
+// round-1 pacer) instead of in bursts (A/B measurements).
 bool burst_pacing_enabled() {
   static const bool on = [] {
     const char* e = getenv("WIND_KV_BURST_PACING");
@@ -1240,7 +1240,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     grid = std::min<int64_t>(grid, to_host ? ctas_for_in_flight(kHostToHostInFlight, ring) : kHostCtasFromHost);
   }
   // Rate limits.  Device ops (INTRA / PEER) with no CTA cap are BURST-paced: the op is cut
-  // into slices of its units, each slice moved by the full grid at full rate and followed
+  // into slices of its units, each slice moved by half the grid at full rate and followed
   // by a 1-thread pace kernel that holds the stream until the rate schedule allows the next
   // one (2 ms of rate budget per slice).  Between bursts no copy CTA is resident, so a
   // co-running decode step keeps every SM: a paced grid of sleeping CTAs (the round-1
