@@ -1143,6 +1143,47 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None, victim_
             "victim_ms_alone_adjacent": round(tr, 3), "victim_ms_with_migration": round(tw, 3),
             "slowdown": round(tw / tr - 1.0, 4),
             "note": "one full-rate op per decode step, released at the step's start"}
+    # The library's step-aligned op (wind_kv_migrate_stepped): slices released by the
+    # victim's own step signal (wind_kv_step_signal before each step's graph replay), the
+    # whole migration enqueued up front on the low-priority stream.
+    counter = torch.zeros(1, dtype=torch.int32, device=dev)
+    issued = [0]
+    for avg in (50, 150):
+        bps = int(avg * 1e9 * t_alone * 1e-3)
+
+        def stepped_run(n):
+            base, k = issued[0], 0
+            while k < n:
+                n0 = wk.launch_count()
+                wk.migrate_stepped(src, d_tabs[0], dst, d_tabs[1], counter, first_step=base + k + 1,
+                                   bytes_per_step=bps, n=case.n, stream=lo_s)
+                k += wk.launch_count() - n0
+            ev = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
+            ev[0].record(hi_s)
+            for i in range(n):
+                wk.step_signal(counter, stream=hi_s)
+                with torch.cuda.stream(hi_s):
+                    graph.replay()
+                ev[i + 1].record(hi_s)
+            for _ in range(k - n):  # release the slices enqueued past the last step
+                wk.step_signal(counter, stream=hi_s)
+            issued[0] = base + k
+            return ev
+        alone_s, with_s = [], []
+        for _ in range(rounds):
+            torch.cuda.synchronize()
+            ev = victim_run(n_round)
+            torch.cuda.synchronize()
+            alone_s += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
+            ev = stepped_run(n_round)
+            torch.cuda.synchronize()
+            with_s += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
+        tr, tw = float(np.median(alone_s)), float(np.median(with_s))
+        res[f"stepped_avg{avg}GBs"] = {
+            "bytes_per_step": bps, "avg_gbs": round(bps / tr / 1e6, 1),
+            "victim_ms_alone_adjacent": round(tr, 3), "victim_ms_with_migration": round(tw, 3),
+            "slowdown": round(tw / tr - 1.0, 4),
+            "note": "wind_kv_migrate_stepped: slices released by the victim's wind_kv_step_signal"}
     clk.__exit__()
     wk.set_tuning(wk.PATH_INTRA, **saved)
     wk.set_tuning(wk.PATH_HOST, **saved_host)

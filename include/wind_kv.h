@@ -270,6 +270,30 @@ wind_status wind_kv_migrate_batch(const wind_kv_pool* src, const wind_kv_migrate
 wind_status wind_kv_route(const wind_kv_pool* src, const wind_kv_pool* dst, int32_t* exec_device,
                           int32_t* path, int32_t* sys_scope);
 
+/* Step-aligned migrate (interference, S§8(d); DESIGN.md §6 "burst instead of trickle"):
+ * the op of wind_kv_migrate, cut into slices of about `bytes_per_step` payload bytes (work
+ * units in layer-ascending order); slice k waits on `stream` until *step_counter >=
+ * first_step + k (wrap-safe, cuStreamWaitValue32 GEQ) and then runs at full rate on half
+ * the grid.  The consumer's decode loop calls wind_kv_step_signal(step_counter, its
+ * stream) at the start of every decode step, so each slice overlaps the beginning of one
+ * decode step instead of trickling through all of them (next to an HBM-saturating decode
+ * step: ~1.4 % at 50 GB/s and ~4.5 % at 150 GB/s average, against 4-5 % / 7-23 % for rate
+ * limits).  `first_step` is the counter value of the step that releases slice 0 (the caller
+ * knows its step count; inside a CUDA graph the waits are constants of the graph).
+ * Results, tickets and layer flags are those of wind_kv_migrate (one op: a layer is
+ * published when its last slice has landed).  step_counter: device-accessible uint32,
+ * 4-byte aligned, owned by the caller.  Errors: as wind_kv_migrate, plus INVALID_ARG (NULL
+ * or misaligned counter, bytes_per_step == 0) and UNSUPPORTED (host pools, debug pools,
+ * copy-engine kernels).  The op never completes if the consumer stops signalling. */
+wind_status wind_kv_migrate_stepped(const wind_kv_pool* src, const int32_t* src_bt, wind_kv_pool* dst,
+                                    const int32_t* dst_bt, int32_t n_blocks, int32_t layer_lo,
+                                    int32_t layer_hi, const uint32_t* step_counter, uint32_t first_step,
+                                    uint64_t bytes_per_step, void* stream);
+
+/* Adds 1 to *step_counter on `stream` (device side, release at GPU scope, in stream order):
+ * the consumer's "a decode step starts here" for wind_kv_migrate_stepped. */
+wind_status wind_kv_step_signal(uint32_t* step_counter, void* stream);
+
 /* ------------------------------------------------------------- layer flags (A5) */
 
 /* Number of ops this process has enqueued into `dst` so far (the ticket of the latest). */

@@ -20,7 +20,7 @@ import numpy as np
 
 __all__ = [
     "WindKVError", "Pool", "lib", "migrate", "migrate_batch", "migrate_heads", "swap_out", "swap_in", "compact",
-    "layer_wait", "route", "validate", "plan_compact", "plan_rebalance", "check_device_error",
+    "layer_wait", "route", "migrate_stepped", "step_signal", "validate", "plan_compact", "plan_rebalance", "check_device_error",
     "set_tuning", "get_tuning", "launch_count", "STATUS", "PATH_INTRA", "PATH_PEER", "PATH_HOST",
     "KERNEL_AUTO", "KERNEL_TMA", "KERNEL_SIMT", "EXPORTED_SYMBOLS", "Partition",
 ]
@@ -53,6 +53,7 @@ EXPORTED_SYMBOLS = [
     "wind_kv_get_tuning", "wind_kv_migrate_ex", "wind_kv_launch_count", "wind_kv_status_string",
     "wind_kv_last_error",
     "wind_kv_version", "wind_kv_partition_sms", "wind_kv_partition_destroy", "wind_kv_route",
+    "wind_kv_migrate_stepped", "wind_kv_step_signal",
 ]
 
 
@@ -130,6 +131,8 @@ def lib() -> ct.CDLL:
         "wind_kv_partition_sms": [I32, I32, ct.POINTER(SmPartition)],
         "wind_kv_partition_destroy": [ct.POINTER(SmPartition)],
         "wind_kv_route": [P, P, ct.POINTER(I32), ct.POINTER(I32), ct.POINTER(I32)],
+        "wind_kv_migrate_stepped": [P, P, P, P, I32, I32, I32, P, U32, ct.c_uint64, P],
+        "wind_kv_step_signal": [P, P],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -383,6 +386,26 @@ def compact(pool: Pool, src_bt, dst_bt, n: Optional[int] = None, stream=None) ->
     n = _len(src_bt) if n is None else n
     _check(lib().wind_kv_compact(pool.handle, _ptr(src_bt), _ptr(dst_bt), n,
                                  _stream(stream, pool.device)))
+
+
+def migrate_stepped(src: Pool, src_bt, dst: Pool, dst_bt, step_counter, first_step: int,
+                    bytes_per_step: int, n: Optional[int] = None, layer_lo: Optional[int] = None,
+                    layer_hi: Optional[int] = None, stream=None) -> None:
+    """wind_kv_migrate_stepped: the migrate cut into ~bytes_per_step slices, slice k released
+    when the int32/uint32 device tensor (or address) `step_counter` reaches first_step + k."""
+    n = _len(src_bt) if n is None else n
+    lo = max(src.layers[0], dst.layers[0]) if layer_lo is None else layer_lo
+    hi = min(src.layers[1], dst.layers[1]) if layer_hi is None else layer_hi
+    cp = step_counter if isinstance(step_counter, int) else step_counter.data_ptr()
+    _check(lib().wind_kv_migrate_stepped(src.handle, _ptr(src_bt), dst.handle, _ptr(dst_bt), n, lo, hi, cp,
+                                         first_step, bytes_per_step, _stream(stream, _exec_device(src, dst))))
+
+
+def step_signal(step_counter, stream=None) -> None:
+    """wind_kv_step_signal: +1 on the step counter, in stream order (a decode step starts)."""
+    cp = step_counter if isinstance(step_counter, int) else step_counter.data_ptr()
+    dev = 0 if isinstance(step_counter, int) else step_counter.device.index
+    _check(lib().wind_kv_step_signal(cp, _stream(stream, dev)))
 
 
 def route(src: Pool, dst: Pool) -> tuple[int, int, bool]:

@@ -879,8 +879,17 @@ wind_status copy_engine_op(const Params& p, int32_t src_nb, const OpItem* items,
   return WIND_OK;
 }
 
+// Step-aligned pacing (wind_kv_migrate_stepped): slice k of the op waits until
+// *counter >= first + k, the consumer's decode loop bumping the counter at each step start.
+struct StepPacing {
+  const uint32_t* counter;
+  uint32_t first;
+  uint64_t bytes_per_step;
+};
+
 wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
-                   int32_t hi, void* stream, const HeadRange& hr, const wind_kv_tuning* override_tuning);
+                   int32_t hi, void* stream, const HeadRange& hr, const wind_kv_tuning* override_tuning,
+                   const StepPacing* step);
 
 // Staged copy-engine host path (kernel 4, opt-in: the host-side block table is read on the
 // CPU at enqueue, unlike every other op's tables).  PCIe is the bottleneck of a swap, and the DMA
@@ -1017,7 +1026,7 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
     if (out) {
       if (k >= g.nbufs) WKV_CUDA(cudaStreamWaitEvent(s, g.freed[b], 0), "cudaStreamWaitEvent(freed)");
       OpItem gi{&stage, dev_bt + i0, g.iota, mk};
-      if ((st = run_op(dev, &gi, 1, la, lb, s, HeadRange(), k == 0 ? &t_exposed : &t_hidden)) != WIND_OK)
+      if ((st = run_op(dev, &gi, 1, la, lb, s, HeadRange(), k == 0 ? &t_exposed : &t_hidden, nullptr)) != WIND_OK)
         return st;
       cudaStream_t ds = g.side[k % nside];
       WKV_CUDA(cudaEventRecord(g.ready[b], s), "cudaEventRecord(ready)");
@@ -1036,7 +1045,7 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
       WKV_CUDA(cudaEventRecord(g.ready[b], g.side[0]), "cudaEventRecord(ready)");
       WKV_CUDA(cudaStreamWaitEvent(s, g.ready[b], 0), "cudaStreamWaitEvent(ready)");
       OpItem si{&shadow, g.iota, dev_bt + i0, mk};
-      if ((st = run_op(&stage, &si, 1, la, lb, s, HeadRange(), k == K - 1 ? &t_exposed : &t_hidden)) != WIND_OK)
+      if ((st = run_op(&stage, &si, 1, la, lb, s, HeadRange(), k == K - 1 ? &t_exposed : &t_hidden, nullptr)) != WIND_OK)
         return st;
       if (layers_done && (st = flag_range(la, lb, s)) != WIND_OK) return st;
       WKV_CUDA(cudaEventRecord(g.freed[b], s), "cudaEventRecord(freed)");
@@ -1056,10 +1065,10 @@ wind_status staged_host_op(const wind_kv_pool* src, const OpItem& it, int32_t lo
 // The common op: src -> items[] over layers [lo, hi) on `stream`.
 wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
                    int32_t hi, void* stream, const HeadRange& hr = HeadRange(),
-                   const wind_kv_tuning* override_tuning = nullptr);
+                   const wind_kv_tuning* override_tuning = nullptr, const StepPacing* step = nullptr);
 wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, int32_t lo,
                    int32_t hi, void* stream, const HeadRange& hr,
-                   const wind_kv_tuning* override_tuning) {
+                   const wind_kv_tuning* override_tuning, const StepPacing* step) {
   if (!src) return fail(WIND_ERR_INVALID_ARG, "src pool is NULL");
   if (n_items < 1 || n_items > WIND_KV_MAX_BATCH) return fail(WIND_ERR_INVALID_ARG, "n_items out of range");
   struct NvtxRange {  // one NVTX range per op (the enqueue, on the host timeline)
@@ -1113,6 +1122,12 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   DeviceGuard g(exec);
 
+  if (step) {  // step-aligned slices: device pools (INTRA / PEER), SM kernels, no debug pools
+    bool dbg = false;
+    for (int j = 0; j < n_items; ++j) dbg = dbg || ((src->desc.flags | items[j].dst->desc.flags) & WIND_POOL_DEBUG);
+    if (path == WIND_PATH_HOST || dbg || t.kernel == kCopyEngine || t.kernel == kStaged)
+      return fail(WIND_ERR_UNSUPPORTED, "step-aligned ops need device pools, an SM kernel and no debug pool");
+  }
   bool debug = false;
   for (int j = 0; j < n_items; ++j)
     if (items[j].n > 0 && ((src->desc.flags | items[j].dst->desc.flags) & WIND_POOL_DEBUG)) {
@@ -1262,12 +1277,13 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   p.unit_lo = 0;
   p.unit_hi = p.total_units;
   p.first_slice = 1;
-  if (burst_paced) {
+  if (burst_paced || step) {
     // source payload of the op (a fan-out reads each unit once)
     int64_t n_src = 0;
     for (int j = 0; j < (fan > 1 ? 1 : n_items); ++j) n_src += items[j].n;
     const double payload = 2.0 * p.n_layers * static_cast<double>(CP) * static_cast<double>(n_src);
-    const double slice_bytes = t.rate_mbps * 1e6 * burst_period_ns() * 1e-9;
+    const double slice_bytes = step ? static_cast<double>(step->bytes_per_step)
+                                    : t.rate_mbps * 1e6 * burst_period_ns() * 1e-9;
     int64_t slice_units = static_cast<int64_t>(p.total_units * slice_bytes / std::max(1.0, payload));
     // a burst runs on half the grid: nearly the full HBM rate (one CTA moves ~38 GB/s), and
     // half the SMs stay with the co-running work (sweep, profiles/r02/burst_pacer/: 74 CTAs
@@ -1279,16 +1295,28 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     slice_units = std::max<int64_t>(slice_units, grid);  // a burst keeps the whole grid busy
     unsigned long long* t0 = ctx->stamps + slot;
     p.ns_per_byte = 0.f;
-    WKV_CUDA(launch_pace(t0, 0, 1, s), "pace kernel launch");
-    int launches = 1;
-    for (int64_t u = 0; u < p.total_units; u += slice_units) {
+    static PFN_waitValue32 wait_fn = driver_fn<PFN_waitValue32>("cuStreamWaitValue32");
+    if (step && !wait_fn) return fail(WIND_ERR_CUDA, "cuStreamWaitValue32 entry point unavailable");
+    int launches = 0;
+    if (!step) {
+      WKV_CUDA(launch_pace(t0, 0, 1, s), "pace kernel launch");
+      ++launches;
+    }
+    uint32_t k = 0;
+    for (int64_t u = 0; u < p.total_units; u += slice_units, ++k) {
       p.unit_lo = u;
       p.unit_hi = std::min<int64_t>(p.total_units, u + slice_units);
       p.first_slice = u == 0;
+      if (step) {  // released by the consumer's step `first + k` (wrap-safe >=)
+        CUresult r = wait_fn(static_cast<CUstream>(stream), reinterpret_cast<CUdeviceptr>(step->counter),
+                             step->first + k, CU_STREAM_WAIT_VALUE_GEQ);
+        if (r != CUDA_SUCCESS) return fail(WIND_ERR_CUDA, "cuStreamWaitValue32 failed (CUresult %d)", static_cast<int>(r));
+      }
       cudaError_t e = launch_copy(p, kernel, static_cast<int>(std::min<int64_t>(grid, p.unit_hi - u)), s,
                                   pdl_enabled());
       if (e != cudaSuccess) return cuda_fail(e, "copy kernel launch");
       ++launches;
+      if (step) continue;
       // hold the stream until the schedule reaches the bytes moved so far (after the last
       // slice too: the op then ends when its rate says, as the in-kernel pacer's ops do)
       const double done = payload * static_cast<double>(p.unit_hi) / static_cast<double>(p.total_units);
@@ -1577,6 +1605,36 @@ extern "C" wind_status wind_kv_migrate_ex(const wind_kv_pool* src, const int32_t
   }
   OpItem it{dst, src_bt, dst_bt, n_blocks};
   return run_op(src, &it, 1, layer_lo, layer_hi, stream, HeadRange(), tuning);
+}
+
+extern "C" wind_status wind_kv_migrate_stepped(const wind_kv_pool* src, const int32_t* src_bt,
+                                               wind_kv_pool* dst, const int32_t* dst_bt, int32_t n_blocks,
+                                               int32_t layer_lo, int32_t layer_hi,
+                                               const uint32_t* step_counter, uint32_t first_step,
+                                               uint64_t bytes_per_step, void* stream) {
+  if (!dst) return fail(WIND_ERR_INVALID_ARG, "dst pool is NULL");
+  if (!step_counter || bytes_per_step == 0)
+    return fail(WIND_ERR_INVALID_ARG, "step_counter is NULL or bytes_per_step is 0");
+  if (reinterpret_cast<uintptr_t>(step_counter) & 3) return fail(WIND_ERR_INVALID_ARG, "step_counter misaligned");
+  OpItem it{dst, src_bt, dst_bt, n_blocks};
+  const StepPacing sp{step_counter, first_step, bytes_per_step};
+  return run_op(src, &it, 1, layer_lo, layer_hi, stream, HeadRange(), nullptr, &sp);
+}
+
+extern "C" wind_status wind_kv_step_signal(uint32_t* step_counter, void* stream) {
+  if (!step_counter || (reinterpret_cast<uintptr_t>(step_counter) & 3))
+    return fail(WIND_ERR_INVALID_ARG, "step_counter is NULL or misaligned");
+  int d = -1;  // load the library's kernels on the stream's device first (no lazy loading later)
+  if (!stream || cudaStreamGetDevice(static_cast<cudaStream_t>(stream), &d) != cudaSuccess) {
+    cudaGetLastError();
+    WKV_CUDA(cudaGetDevice(&d), "cudaGetDevice");
+  }
+  DevCtx* ctx;
+  wind_status st = dev_ctx(d, &ctx);
+  if (st != WIND_OK) return st;
+  WKV_CUDA(launch_step_signal(step_counter, static_cast<cudaStream_t>(stream)), "step signal launch");
+  g_launches += 1;
+  return WIND_OK;
 }
 
 extern "C" wind_status wind_kv_get_tuning(int32_t path, wind_kv_tuning* t) {

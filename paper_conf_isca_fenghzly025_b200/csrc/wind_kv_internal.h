@@ -78,6 +78,9 @@ cudaError_t launch_flag_bump(const Params& p, cudaStream_t s);
 // launches sleep until *t0 + target_ns.
 cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s);
 
+// wind_kv_step_signal: +1 on a consumer's step counter (release, GPU scope), in stream order.
+cudaError_t launch_step_signal(uint32_t* counter, cudaStream_t s);
+
 // Launchers (wind_kv_kernels.cu).  Return cudaGetLastError() after the launch.
 // pdl: launch with programmatic stream serialization (the kernel's prologue may overlap the
 // previous kernel on the stream; it waits for it before touching global memory).

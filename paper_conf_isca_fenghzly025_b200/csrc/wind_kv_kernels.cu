@@ -636,6 +636,13 @@ __global__ void pace_kernel(unsigned long long* t0, uint64_t target_ns, int firs
   }
 }
 
+// Step-aligned ops (wind_kv_migrate_stepped): the consumer's decode loop bumps its step
+// counter at each step start; slices of a stepped op wait on it with cuStreamWaitValue32.
+// A release reduction: the work before it on the stream is visible before the new count.
+__global__ void step_signal_kernel(uint32_t* counter) {
+  asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(counter) : "memory");
+}
+
 // -------------------------------------------------------- debug-pool device table check
 
 __global__ void table_count_kernel(const int32_t* sbt, const int32_t* dbt, int32_t n,
@@ -679,6 +686,7 @@ cudaError_t prepare_kernels(int device, size_t max_tma_smem) {
   // of a kernel loads its code, which synchronises the whole device — an op must never do
   // that on the hot path.
   const void* fns[] = {reinterpret_cast<const void*>(simt_copy_kernel),
+                       reinterpret_cast<const void*>(step_signal_kernel),
                        reinterpret_cast<const void*>(flag_bump_kernel),
                        reinterpret_cast<const void*>(pace_kernel),
                        reinterpret_cast<const void*>(table_count_kernel),
@@ -711,6 +719,11 @@ cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s, b
 
 cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s) {
   pace_kernel<<<1, 1, 0, s>>>(t0, target_ns, first);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_step_signal(uint32_t* counter, cudaStream_t s) {
+  step_signal_kernel<<<1, 1, 0, s>>>(counter);
   return cudaGetLastError();
 }
 

@@ -280,3 +280,58 @@ def test_ops_enqueued_from_many_host_threads():
         for p, w in zip(pools, want):
             np.testing.assert_array_equal(p.tensor().cpu().numpy(), w)
             assert p.layer_ticket() == 10 and [p.layer_count(l) for l in range(L)] == [10] * L
+
+
+def test_migrate_stepped_releases_slices_per_step():
+    """wind_kv_migrate_stepped: the op is cut into slices released one per consumer step
+    (wind_kv_step_signal): nothing moves before the first signal; after enough signals the
+    whole pool equals the oracle, every layer flag moved exactly once, one ticket."""
+    import time
+    import oracle as O
+    from windgen import SHAPES
+    sh = SHAPES["C2"]
+    L, nb, n = 6, 160, 120
+    src = wk.Pool(L, sh.n_kv_heads, sh.head_dim, 16, 2, nb)
+    dst = wk.Pool(L, sh.n_kv_heads, sh.head_dim, 16, 2, nb)
+    rng = np.random.default_rng(9)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    d0 = rng.integers(0, 256, dst.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    dst.tensor().copy_(torch.from_numpy(d0))
+    sbt = rng.permutation(nb)[:n].astype(np.int32)
+    dbt = rng.permutation(nb)[:n].astype(np.int32)
+    ts, td = torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)
+    counter = torch.zeros(1, dtype=torch.int32, device=DEV)
+    mig, dec = torch.cuda.Stream(DEV), torch.cuda.Stream(DEV)
+    payload = 2 * L * n * sh.chunk_bytes  # 225 MiB -> 5 slices of ~48 MB
+    torch.cuda.synchronize()
+    n0 = wk.launch_count()
+    wk.migrate_stepped(src, ts, dst, td, counter, first_step=1, bytes_per_step=payload // 5 + 1, stream=mig)
+    slices = wk.launch_count() - n0
+    assert 4 <= slices <= 6 and dst.layer_ticket() == 1
+    time.sleep(0.05)
+    assert not mig.query()  # blocked on step 1
+    np.testing.assert_array_equal(dst.tensor().cpu().numpy(), d0)  # nothing moved yet
+    for _ in range(slices):
+        wk.step_signal(counter, stream=dec)
+        dec.synchronize()
+    mig.synchronize()
+    assert int(counter.item()) == slices
+    want = d0.copy()
+    g = O.Geom(0, L, sh.n_kv_heads, sh.head_dim, 16, 2, nb)
+    assert O.migrate(s0, g, sbt, want, g, dbt, 0, L) == O.OK
+    np.testing.assert_array_equal(dst.tensor().cpu().numpy(), want)
+    assert [dst.layer_count(l) for l in range(L)] == [1] * L
+    # argument errors, nothing enqueued
+    n1 = wk.launch_count()
+    for bad in (dict(step_counter=0), dict(bytes_per_step=0)):
+        kw = dict(step_counter=counter, first_step=1, bytes_per_step=1 << 20)
+        kw.update(bad)
+        with pytest.raises(wk.WindKVError) as e:
+            wk.migrate_stepped(src, ts, dst, td, stream=mig, **kw)
+        assert e.value.status == -1
+    host = wk.Pool(L, sh.n_kv_heads, sh.head_dim, 16, 2, nb, loc="host")
+    with pytest.raises(wk.WindKVError) as e:
+        wk.migrate_stepped(src, ts, host, td, counter, 1, 1 << 20, stream=mig)
+    assert e.value.status == -10
+    assert wk.launch_count() == n1 and dst.layer_ticket() == 1
