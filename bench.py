@@ -799,22 +799,16 @@ def run_stall_free(wk, device, cap_ctas: int = 16) -> dict:
                 "pause_ms": round(resb.pause_ms, 3), "blocks_sent": resb.blocks_sent}}
 
 
-def run_interference(wk, device, peaks, n_victim_steps=50, configs=None, victim_kind="attention") -> dict:
-    """S§8(d) interference, C3 (OPT-66B KV, 64 layers x 72 heads x d 128, fp16): the victim
-    is paged decode attention over 16 x 2048 resident tokens (the Fig. 8 decode set,
-    P:251) = 72 GiB of KV read per step (64 layer launches) on a HIGH-priority stream; the
-    migration moves 4 x 2048-token long-context requests (P:227, 18 GiB) on a LOW-priority
-    side stream, looped to cover every victim step.  On one GPU the migration is
-    intra-device (reads AND writes this HBM); a CTA cap emulates the source-side HBM load
-    of an NVLink push (8 CTAs ~ 365 GB/s payload = 730 GB/s of DRAM traffic, about what a
-    770 GB/s peer push reads on its source GPU).
-
-    victim_kind="decode_step": a victim closer to a whole decode step of OPT-66B on one
-    TP-2 rank (Table 3 placements are TP-2, P:301-308): per layer the QKV projection, paged
-    attention over this rank's 36 heads of the 16 x 2048-token set, the output projection
-    and the MLP — fp16 GEMMs (cuBLAS, harness only) against one layer's weight shard
-    (1.02 GB, re-read every layer: it cannot stay in the 126 MB L2) — so a step streams
-    65 GB of weights plus 36 GiB of KV."""
+def make_victim(wk, device, peaks, victim_kind="attention", n_steps=50):
+    """The co-running decode work of the interference measurements (S§8(d)), as one CUDA
+    graph per step on a HIGH-priority stream (plus a LOW-priority stream for the migration):
+    "attention" = paged decode attention over 16 x 2048 resident tokens of OPT-66B KV (the
+    Fig. 8 decode set; 72 GiB read per step), "decode_step" = a whole OPT-66B decode
+    step on one TP-2 rank (QKV, attention over 36 heads, output projection, MLP; fp16 cuBLAS
+    GEMMs on one layer's 1.02 GB weight shard re-read every layer).  Returns a namespace
+    with the graph, the streams, run(n) (per-step events), step_on(stream) (to capture it
+    elsewhere), t_alone (median step ms) and info (description, HBM fraction)."""
+    import types
     import torch
     import victim
     from windgen import migration_case, SHAPES, KVShape
@@ -893,18 +887,46 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None, victim_
                 g.replay()
                 ev[i + 1].record(st)
         return ev
-    ev = victim_run(n_victim_steps)
+    ev = victim_run(n_steps)
     torch.cuda.synchronize()
-    alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_victim_steps)]
+    alone = [ev[i].elapsed_time(ev[i + 1]) for i in range(n_steps)]
     t_alone = float(np.median(alone))
     kv_read = B * ctx_len * sh.n_layers * 2 * hv * sh.head_dim * sh.elem_bytes
     step_bytes = kv_read + (w_bytes * sh.n_layers if full_step else 0)
-    res = {"victim_ms_alone": round(t_alone, 3),
+    info = {"victim_ms_alone": round(t_alone, 3),
            "victim_hbm_frac": round(step_bytes / t_alone / 1e6 / peaks["hbm_gbs"], 3),
            "victim": ("OPT-66B decode step on one TP-2 rank: QKV, paged attention (36 heads, "
                       "16 x 2048 tok), output projection, MLP; 64 layers; weights "
                       f"{w_bytes * sh.n_layers / 1e9:.1f} GB + KV {kv_read / 1e9:.1f} GB per step"
                       if full_step else "paged decode attention, 16 x 2048 tok, 64 layers, 72 heads (C3)")}
+
+    return types.SimpleNamespace(graph=graph, hi_s=hi_s, lo_s=lo_s, run=victim_run, step_on=victim_step_on,
+                                 t_alone=t_alone, info=info, pool=vpool, sh=sh, dev=dev)
+
+
+def run_interference(wk, device, peaks, n_victim_steps=50, configs=None, victim_kind="attention") -> dict:
+    """S§8(d) interference, C3 (OPT-66B KV, 64 layers x 72 heads x d 128, fp16): the victim
+    is paged decode attention over 16 x 2048 resident tokens (the Fig. 8 decode set,
+    P:251) = 72 GiB of KV read per step (64 layer launches) on a HIGH-priority stream; the
+    migration moves 4 x 2048-token long-context requests (P:227, 18 GiB) on a LOW-priority
+    side stream, looped to cover every victim step.  On one GPU the migration is
+    intra-device (reads AND writes this HBM); a CTA cap emulates the source-side HBM load
+    of an NVLink push (8 CTAs ~ 365 GB/s payload = 730 GB/s of DRAM traffic, about what a
+    770 GB/s peer push reads on its source GPU).
+
+    victim_kind="decode_step": a victim closer to a whole decode step of OPT-66B on one
+    TP-2 rank (Table 3 placements are TP-2, P:301-308): per layer the QKV projection, paged
+    attention over this rank's 36 heads of the 16 x 2048-token set, the output projection
+    and the MLP — fp16 GEMMs (cuBLAS, harness only) against one layer's weight shard
+    (1.02 GB, re-read every layer: it cannot stay in the 126 MB L2) — so a step streams
+    65 GB of weights plus 36 GiB of KV."""
+    import torch
+    from windgen import migration_case
+    V = make_victim(wk, device, peaks, victim_kind, n_victim_steps)
+    sh, dev = V.sh, V.dev
+    graph, hi_s, lo_s, victim_step_on, victim_run, t_alone = V.graph, V.hi_s, V.lo_s, V.step_on, V.run, V.t_alone
+    full_step = victim_kind == "decode_step"
+    res = dict(V.info)
 
     case = migration_case("C3")
     src = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
@@ -1191,7 +1213,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None, victim_
     for P, _ in part.values():
         P.destroy()
     host.destroy()
-    del vpool, src, dst, sink
+    del V, src, dst, sink
     return res
 
 
@@ -1265,7 +1287,111 @@ def run_all_to_all(wk, rank, world, device, peaks, steps=5, warmup=3, scale=1.0)
     return out
 
 
-# -------------------------------------------------------------------------- main
+def run_peer_interference(wk, rank, world, device, peaks, rounds=3, n_steps=20) -> dict:
+    """Interference on the REAL multi-GPU configuration (S§8(d); "decoding continues
+    during migration"): every rank runs the whole-decode-step victim (make_victim
+    "decode_step") while the prefill rank of each pair pushes C3 long-context KV into
+    its partner's imported pool over NVLink — trickled at 150 GB/s (the burst pacer),
+    uncapped, or as wind_kv_migrate_stepped slices released by the SOURCE rank's own decode
+    steps (avg 150 / 400 GB/s).  Reported per side: the source (push) rank's victim reads
+    only (its HBM serves the push's loads), the destination rank's victim sees the push's
+    writes.  Each configuration is measured against an adjacent victim-alone run; slowdowns
+    are the max over pairs.  With every rank on one GPU (WIND_BENCH_ONE_DEVICE) the code path
+    runs but the numbers are not NVLink numbers."""
+    import threading
+    import torch
+    import torch.distributed as dist
+    from paper_conf_isca_fenghzly025_b200 import parallel
+    from windgen import migration_case
+    role, partner = parallel.pair_role(rank, world)
+    V = make_victim(wk, device, peaks, "decode_step", n_steps)
+    dev = torch.device("cuda", device)
+    case = migration_case("C3")
+    sh = case.shape
+    src = dst = None
+    if role == "push":
+        src = make_pool(wk, sh, case.nb_src, device, case.content_seed, case.src_tag)
+    if role == "decode":
+        dst = make_pool(wk, sh, case.nb_dst, device, case.content_seed, case.dst_tag)
+    handles = parallel.exchange_handles(dst.export() if role == "decode" else None)
+    if role == "push":
+        dst = wk.Pool.import_(handles[partner], device)
+    sbt, dbt = torch.as_tensor(case.src_bt, device=dev), torch.as_tensor(case.dst_bt, device=dev)
+    pb = payload_bytes(case.n, sh.n_layers, sh.chunk_bytes)
+    counter = torch.zeros(1, dtype=torch.int32, device=dev)
+    issued = [0]
+
+    path = wk.route(src, dst)[1] if role == "push" else wk.PATH_PEER  # PEER across GPUs
+    saved = wk.get_tuning(path)
+
+    def victim_with(kind, arg):
+        """Runs n_steps of the victim on every rank; the push rank migrates alongside.
+        Returns this rank's per-step ms."""
+        stop, th = threading.Event(), None
+        if role == "push" and kind in ("trickle", "uncapped"):
+            wk.set_tuning(path, **{**saved, "rate_mbps": arg if kind == "trickle" else 0, "max_ctas": 0})
+
+            def feeder():
+                while not stop.is_set():
+                    wk.migrate(src, sbt, dst, dbt, n=case.n, stream=V.lo_s)
+                    V.lo_s.synchronize()
+            th = threading.Thread(target=feeder, daemon=True)
+            th.start()
+            time.sleep(0.01)
+        extra = 0
+        if role == "push" and kind == "stepped":
+            bps, k, base = int(arg * 1e6 * V.t_alone * 1e-3), 0, issued[0]
+            while k < n_steps:
+                n0 = wk.launch_count()
+                wk.migrate_stepped(src, sbt, dst, dbt, counter, first_step=base + k + 1, bytes_per_step=bps,
+                                   n=case.n, stream=V.lo_s)
+                k += wk.launch_count() - n0
+            extra = k - n_steps
+            issued[0] = base + k
+        ev = [torch.cuda.Event(enable_timing=True) for _ in range(n_steps + 1)]
+        ev[0].record(V.hi_s)
+        for i in range(n_steps):
+            if role == "push" and kind == "stepped":
+                wk.step_signal(counter, stream=V.hi_s)
+            with torch.cuda.stream(V.hi_s):
+                V.graph.replay()
+            ev[i + 1].record(V.hi_s)
+        for _ in range(extra):
+            wk.step_signal(counter, stream=V.hi_s)
+        V.hi_s.synchronize()
+        stop.set()
+        if th is not None:
+            th.join()
+        torch.cuda.synchronize()
+        wk.set_tuning(path, **saved)
+        return [ev[i].elapsed_time(ev[i + 1]) for i in range(n_steps)]
+
+    out = {"victim": V.info["victim"], "victim_ms_alone": V.info["victim_ms_alone"], "pairs": world // 2}
+    for name, kind, arg in (("trickle150GBs", "trickle", 150000), ("uncapped", "uncapped", 0),
+                            ("stepped_avg150GBs", "stepped", 150000), ("stepped_avg400GBs", "stepped", 400000)):
+        alone, withm = [], []
+        for _ in range(rounds):
+            dist.barrier()
+            alone += victim_with("alone", 0)
+            dist.barrier()
+            withm += victim_with(kind, arg)
+        slow = float(np.median(withm)) / float(np.median(alone)) - 1.0
+        # per side: max over the ranks of that role
+        sides = [None] * world
+        dist.all_gather_object(sides, (role, slow))
+        src_s = [x for r, x in sides if r == "push"]
+        dst_s = [x for r, x in sides if r == "decode"]
+        out[name] = {"source_slowdown": round(max(src_s), 4) if src_s else None,
+                     "destination_slowdown": round(max(dst_s), 4) if dst_s else None}
+    out["payload_gib_per_op"] = round(pb / GiB, 2)
+    if role == "push":
+        dst.destroy()
+    dist.barrier()
+    del V, src, dst
+    return out
+
+
+# -------------------------------------------------------------------------- main# -------------------------------------------------------------------------- main
 
 def run_gpu(args) -> None:
     import torch
@@ -1417,6 +1543,7 @@ def run_gpu(args) -> None:
     total_bytes = pb * n_movers
     a2a = None
     compaction = None
+    peer_interf = None
     scen_error = None
     if world > 1 and args.scenarios:
         # The multi-GPU scenarios never ran on more than one GPU in round 1 (one GPU per
@@ -1434,6 +1561,10 @@ def run_gpu(args) -> None:
             ms_c, = parallel.max_over_ranks([msc])
             compaction = {"aggregate_gbs": round(float(tot_b.item()) / ms_c / 1e6, 1), "ms_max": round(ms_c, 3),
                           "hbm_frac_per_gpu": round(2 * float(tot_b.item()) / world / ms_c / 1e6 / peaks["hbm_gbs"], 3)}
+            torch.cuda.empty_cache()
+            # the co-running decode step on the source and destination GPUs of NVLink pushes
+            if args.peer_interference:
+                peer_interf = run_peer_interference(wk, rank, world, local, peaks)
         except Exception as e:  # noqa: BLE001 — reported, not swallowed
             scen_error = f"{type(e).__name__}: {e}"[:400]
             print(f"[bench rank {rank}] multi-GPU scenario failed: {scen_error}", file=sys.stderr, flush=True)
@@ -1461,7 +1592,8 @@ def run_gpu(args) -> None:
         if peer_tune is not None:
             extra["peer_autotune"] = peer_tune
         if a2a is not None or scen_error is not None:
-            extra["scenarios"] = {"c5_all_to_all": a2a, "c5_compaction_all_ranks": compaction}
+            extra["scenarios"] = {"c5_all_to_all": a2a, "c5_compaction_all_ranks": compaction,
+                                  "c3_peer_interference": peer_interf}
             if scen_error is not None:
                 extra["scenarios"]["error"] = scen_error
         if world == 1 and not args.no_cpu_baseline:
@@ -1576,6 +1708,8 @@ def main():
     ap.add_argument("--scenarios", dest="scenarios", action="store_true", default=True)
     ap.add_argument("--no-scenarios", dest="scenarios", action="store_false")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-peer-interference", dest="peer_interference", action="store_false", default=True,
+                    help="N > 1: skip the decode-step victims next to the NVLink pushes (~40 GB per rank)")
     ap.add_argument("--a2a-scale", type=float, default=1.0,
                     help="request-count scale of the N>1 all-to-all scenario (C5 = 1.0)")
     args = ap.parse_args()

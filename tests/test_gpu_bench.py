@@ -45,6 +45,8 @@ def test_bench_multirank_on_one_gpu(world):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={world}",
            "--master-addr", "127.0.0.1", "--master-port", str(_port()), "bench.py", "--gpus", str(world),
            "--steps", "3", "--warmup", "3", "--config", "C1", "--a2a-scale", "0.0625"]
+    if world > 2:  # every rank's ~40 GB decode-step victim on ONE GPU: only at N = 2 here
+        cmd.append("--no-peer-interference")
     out = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
     assert out.returncode == 0, (out.stdout[-2000:], out.stderr[-3000:])
     d = _json_line(out.stdout)
@@ -53,3 +55,10 @@ def test_bench_multirank_on_one_gpu(world):
     assert d["peer_autotune"].get("chosen", "").split("_")[0] in ("push", "pull"), d["peer_autotune"]
     a2a = d["scenarios"]["c5_all_to_all"]
     assert a2a["shuffle"]["blocks_moved"] > 0 and a2a["rebalance"]["aggregate_gbs"] >= 0
+    assert "error" not in d["scenarios"], d["scenarios"].get("error")
+    pi = d["scenarios"]["c3_peer_interference"]
+    if world == 2:  # one pair: both sides measured for every configuration
+        for k in ("trickle150GBs", "uncapped", "stepped_avg150GBs", "stepped_avg400GBs"):
+            assert pi[k]["source_slowdown"] is not None and pi[k]["destination_slowdown"] is not None, pi
+    else:
+        assert pi is None
