@@ -22,6 +22,8 @@ NODES = [
     "tests/test_gpu_parity.py::test_run_coalescing_across_warp_windows",
     "tests/test_gpu_heads.py",
     "tests/test_gpu_fuzz.py",  # 400 random ops (geometry, tables, windows, kernels, swaps)
+    "tests/test_gpu_misc.py::test_burst_paced_op_flags_and_parity",
+    "tests/test_gpu_misc.py::test_migrate_stepped_releases_slices_per_step",
 ]
 
 
