@@ -1258,9 +1258,10 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   // into slices of its units, each slice moved by half the grid at full rate and followed
   // by a 1-thread pace kernel that holds the stream until the rate schedule allows the next
   // one (2 ms of rate budget per slice).  Between bursts no copy CTA is resident, so a
-  // co-running decode step keeps every SM: a paced grid of sleeping CTAs (the round-1
-  // pacer, still used when max_ctas > 0 or on the HOST path) cost a decode step of GEMMs +
-  // attention 19-29 % at 50-150 GB/s, bursts 1.3-4.4 %.
+  // co-running decode step keeps its SMs: at 150 GB/s a paced grid of sleeping CTAs (the
+  // round-1 pacer, still used when max_ctas > 0 or on the HOST path) cost a decode step of
+  // GEMMs + attention 19-29 %, the burst pacer ~7.5 %, and slices released on the
+  // consumer's own steps (wind_kv_migrate_stepped, `step`, same code) ~4.5 %.
   const bool burst_paced = t.rate_mbps > 0 && t.max_ctas == 0 && path != WIND_PATH_HOST && !debug &&
                            burst_pacing_enabled();
   // in-kernel pacing: as few SMs as can sustain the rate (one CTA moves ~38 GB/s of payload
