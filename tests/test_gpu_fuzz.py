@@ -7,7 +7,9 @@ a multiple of the work unit (ragged parts, ragged windows), units smaller than o
 or holding up to 32 chunks, 1-16 token blocks, fp8 / fp16 / fp32 elements, pools whose
 layer windows are shifted (PP stages, `first_layer`), empty and one-block tables, duplicate
 sources (fan-out), same-pool moves with identity pairs, host pools (swap), grids capped
-below the unit count, ring depths 3-8 with every store lag, and the copy-engine path.
+below the unit count, ring depths 3-8 with every store lag, the copy-engine path, and
+(round 2) burst-paced ops and step-released slices (wind_kv_migrate_stepped) of the
+two-pool moves.
 """
 import numpy as np
 import pytest
@@ -107,6 +109,8 @@ def test_random_op_matches_oracle(seed):
     path = wk.PATH_HOST if mode in ("swap_out", "swap_in") else wk.PATH_INTRA
     tuning = draw_tuning(rng, kernel)
     wk.set_tuning(path, **tuning)
+    # device -> device ops with an SM kernel: sometimes burst-paced or step-released slices
+    pace = str(rng.choice(["none", "burst", "stepped"], p=[0.6, 0.2, 0.2])) if mode == "two_pools" else "none"
 
     Hd = int(rng.integers(1, 7)) if mode == "heads" else H   # TP reshard: head counts differ (R24)
     src, s0 = filled(rng, Ls, H, d, bs, eb, nbs, fs, loc=src_loc)
@@ -147,11 +151,28 @@ def test_random_op_matches_oracle(seed):
             wk.swap_out(src, ts, dst, td, n=n)
         elif mode == "swap_in":
             wk.swap_in(src, ts, dst, td, n=n)
+        elif kernel in (wk.KERNEL_TMA, wk.KERNEL_SIMT) and pace != "none" and n > 0 and hi > lo:
+            payload = 2 * (hi - lo) * n * (H * bs * d * eb)
+            k = int(rng.integers(1, 7))  # slices the op is cut into (about)
+            if pace == "burst":  # rate-limited, no CTA cap: slices between pace kernels
+                rate_mbps = max(1, int(payload / k / 2e-3 / 1e6))  # ~k slices of 2 ms budget
+                wk.migrate_ex(src, ts, dst, td, wk.tuning(**{**tuning, "max_ctas": 0, "rate_mbps": rate_mbps}),
+                              n=n, layer_lo=lo, layer_hi=hi)
+            else:  # stepped: slices released by another stream's step signals
+                counter = torch.zeros(1, dtype=torch.int32, device=DEV)
+                s_mig, s_dec = torch.cuda.Stream(DEV), torch.cuda.Stream(DEV)
+                wk.set_tuning(path, **tuning)
+                n0 = wk.launch_count()
+                wk.migrate_stepped(src, ts, dst, td, counter, first_step=1, bytes_per_step=-(-payload // k),
+                                   n=n, layer_lo=lo, layer_hi=hi, stream=s_mig)
+                for _ in range(wk.launch_count() - n0):
+                    wk.step_signal(counter, stream=s_dec)
+                s_mig.synchronize()
         else:
             wk.migrate(src, ts, dst, td, n=n, layer_lo=lo, layer_hi=hi)
     got = read(dst)
     ctx = dict(mode=str(mode), kernel=kernel, tuning=tuning, L=(Ls, Ld), first=(fs, fd), lo=lo, hi=hi,
-               H=(H, Hd), d=d, bs=bs, eb=eb, nb=(nbs, nbd), n=n)
+               H=(H, Hd), d=d, bs=bs, eb=eb, nb=(nbs, nbd), n=n, pace=pace)
     assert np.array_equal(got, want), ctx
     # flags (R19, R23): an op with n > 0 and lo < hi adds exactly 1 to every dst layer flag;
     # an empty op adds nothing
