@@ -73,3 +73,36 @@ def test_full_size_c5_compaction():
     from_src, off = O.expected_origin(g, sbt, g, dbt, 0, sh.n_layers)
     key = windgen.content_key(3005, 7)
     check_all_chunks(pool, from_src, off, sh.chunk_bytes, key, key)
+
+
+@pytest.mark.parametrize("pace", ["stepped", "burst"])
+def test_full_size_c3_paced(pace):
+    """C3 (OPT-66B, 18 GiB) at full size as the round-2 paced forms: wind_kv_migrate_stepped
+    (slices of 2 GiB released by another stream's step signals) and a burst-paced rate
+    limit (2 TB/s: 4 GB slices, ~5 between pace kernels) — every destination chunk vs the
+    oracle's P2 closed form, every layer flag exactly once."""
+    torch.cuda.empty_cache()
+    case = migration_case("C3")
+    sh = case.shape
+    src = pattern_pool(sh, case.nb_src, case.content_seed, case.src_tag)
+    dst = pattern_pool(sh, case.nb_dst, case.content_seed, case.dst_tag)
+    ts, td = torch.as_tensor(case.src_bt, device=DEV), torch.as_tensor(case.dst_bt, device=DEV)
+    s = torch.cuda.Stream(DEV)
+    n0 = wk.launch_count()
+    if pace == "stepped":
+        counter = torch.zeros(1, dtype=torch.int32, device=DEV)
+        wk.migrate_stepped(src, ts, dst, td, counter, first_step=1, bytes_per_step=2 << 30, stream=s)
+        slices = wk.launch_count() - n0
+        assert 8 <= slices <= 10  # 18 GiB / 2 GiB
+        sig = torch.cuda.Stream(DEV)
+        for _ in range(slices):
+            wk.step_signal(counter, stream=sig)
+    else:
+        wk.migrate_ex(src, ts, dst, td, wk.tuning(rate_mbps=2_000_000, max_ctas=0), stream=s)
+        assert 9 <= wk.launch_count() - n0 <= 13  # 1 + 2 x ~5 slices of 4 GB
+    torch.cuda.synchronize()
+    from_src, off = O.expected_origin(geom(src), case.src_bt, geom(dst), case.dst_bt, 0, sh.n_layers)
+    check_all_chunks(dst, from_src, off, sh.chunk_bytes,
+                     windgen.content_key(case.content_seed, case.src_tag),
+                     windgen.content_key(case.content_seed, case.dst_tag))
+    assert all(dst.layer_count(l) == 1 for l in range(sh.n_layers))
