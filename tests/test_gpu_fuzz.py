@@ -129,6 +129,12 @@ def test_random_op_matches_oracle(seed):
         extra = [filled(rng, Ld, H, d, bs, eb, int(rng.integers(n, n + 40)) if n else 1, fd)
                  for _ in range(k - 1)]
         tabs = [dbt] + [rng.permutation(p.desc.n_blocks)[:n].astype(np.int32) for p, _ in extra]
+        if kernel in (wk.KERNEL_TMA, wk.KERNEL_SIMT) and n > 0 and hi > lo and rng.random() < 0.3:
+            # the batch burst-paced: slices of the shared unit space between pace kernels
+            payload = 2 * (hi - lo) * n * (H * bs * d * eb)
+            pace = "burst"
+            wk.set_tuning(path, **{**tuning, "max_ctas": 0,
+                                   "rate_mbps": max(1, int(payload / int(rng.integers(1, 6)) / 2e-3 / 1e6))})
         wk.migrate_batch(src, [(q, ts, to(t), n) for q, t in zip([dst] + [p for p, _ in extra], tabs)], lo, hi)
         for (q, q0), t in zip(extra, tabs[1:]):
             w = q0.copy()
