@@ -1170,14 +1170,15 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None, victim_
     # whole migration enqueued up front on the low-priority stream.
     counter = torch.zeros(1, dtype=torch.int32, device=dev)
     issued = [0]
-    for avg in (50, 150):
+    for avg, proxy in ((50, False), (150, False), (250, True), (400, True)):
         bps = int(avg * 1e9 * t_alone * 1e-3)
+        dpool_, db_ = (sink, zeros_t) if proxy else (dst, d_tabs[1])
 
         def stepped_run(n):
             base, k = issued[0], 0
             while k < n:
                 n0 = wk.launch_count()
-                wk.migrate_stepped(src, d_tabs[0], dst, d_tabs[1], counter, first_step=base + k + 1,
+                wk.migrate_stepped(src, d_tabs[0], dpool_, db_, counter, first_step=base + k + 1,
                                    bytes_per_step=bps, n=case.n, stream=lo_s)
                 k += wk.launch_count() - n0
             ev = [torch.cuda.Event(enable_timing=True) for _ in range(n + 1)]
@@ -1201,7 +1202,7 @@ def run_interference(wk, device, peaks, n_victim_steps=50, configs=None, victim_
             torch.cuda.synchronize()
             with_s += [ev[i].elapsed_time(ev[i + 1]) for i in range(n_round)]
         tr, tw = float(np.median(alone_s)), float(np.median(with_s))
-        res[f"stepped_avg{avg}GBs"] = {
+        res[f"stepped_{'push_source_proxy_' if proxy else ''}avg{avg}GBs"] = {
             "bytes_per_step": bps, "avg_gbs": round(bps / tr / 1e6, 1),
             "victim_ms_alone_adjacent": round(tr, 3), "victim_ms_with_migration": round(tw, 3),
             "slowdown": round(tw / tr - 1.0, 4),
