@@ -134,17 +134,17 @@ wind_status dev_ctx(int dev, DevCtx** out) {
 
 std::mutex g_tune_mu;
 wind_kv_tuning g_tune[3] = {
-    /* INTRA */ {kTma, 1, 49152, 4, 0, 0, 2},  // sweep r01: 0.998 (C2) / 0.985 (C5) of HBM copy
+    /* INTRA */ {kTma, 1, 49152, 4, 0, 0, 2, 0},  // sweep r01: 0.998 (C2) / 0.985 (C5) of HBM copy
     // PEER: SM stores over NVLink (the path the guide measures at 775 GB/s); 96 CTAs of 512
     // threads keep ~3 MiB of stores in flight (> 2 us x 900 GB/s) and leave SMs to the
     // co-running prefill / decode.  Not yet tuned on a multi-GPU box (one GPU per round-1 call).
-    /* PEER  */ {kSimt, 1, 32768, 6, 96, 0, 0},
+    /* PEER  */ {kSimt, 1, 32768, 6, 96, 0, 0, 0},
     // HOST: PCIe-bound.  auto = the TMA kernel on mapped pinned memory (the staged copy-engine
     // path, staged_host_op, is opt-in: kernel 4).
     // max_ctas 0 = per-direction defaults (kHostCtas*): SM stores to host memory beyond
     // what PCIe drains back up into the GPU's memory system — 8 TMA CTAs writing at 52 GB/s
     // slowed a co-running decode kernel by 73 %, 2 CTAs at the same rate by 2 %
-    /* HOST  */ {kAuto, 1, 49152, 4, 0, 0, 2},
+    /* HOST  */ {kAuto, 1, 49152, 4, 0, 0, 2, 0},
 };
 
 // HOST path defaults when the tuning's max_ctas is 0 (sweep r01: scripts/staged_sweep.py and
@@ -428,8 +428,9 @@ extern "C" wind_status wind_kv_pool_create(const wind_kv_pool_desc* desc, void* 
       e = cudaMalloc(&p->base, p->bytes);
       if (e != cudaSuccess) {
         cudaGetLastError();
+        const size_t want = p->bytes;
         delete p;
-        return fail(WIND_ERR_OOM, "cudaMalloc(%zu) failed: %s", p->bytes, cudaGetErrorString(e));
+        return fail(WIND_ERR_OOM, "cudaMalloc(%zu) failed: %s", want, cudaGetErrorString(e));
       }
       p->owns_data = true;
     }
@@ -449,8 +450,9 @@ extern "C" wind_status wind_kv_pool_create(const wind_kv_pool_desc* desc, void* 
       e = cudaHostAlloc(&h, p->bytes, cudaHostAllocMapped | cudaHostAllocPortable);
       if (e != cudaSuccess) {
         cudaGetLastError();
+        const size_t want = p->bytes;
         delete p;
-        return fail(WIND_ERR_OOM, "cudaHostAlloc(%zu) failed: %s", p->bytes, cudaGetErrorString(e));
+        return fail(WIND_ERR_OOM, "cudaHostAlloc(%zu) failed: %s", want, cudaGetErrorString(e));
       }
       void* dptr = nullptr;
       cudaHostGetDevicePointer(&dptr, h, 0);
