@@ -335,3 +335,16 @@ def test_migrate_stepped_releases_slices_per_step():
         wk.migrate_stepped(src, ts, host, td, counter, 1, 1 << 20, stream=mig)
     assert e.value.status == -10
     assert wk.launch_count() == n1 and dst.layer_ticket() == 1
+
+
+def test_pool_larger_than_hbm_is_oom_and_recoverable():
+    """A device pool larger than the GPU's memory: WIND_ERR_OOM with the requested size in
+    the message, nothing leaked, and the next pool creation works (no sticky CUDA error)."""
+    free, _ = torch.cuda.mem_get_info()
+    nb = int(2 * free // (40 * 2 * 40 * 16 * 128 * 2)) + 1  # 2x the free memory, OPT-13B KV blocks
+    with pytest.raises(wk.WindKVError) as e:
+        wk.Pool(40, 40, 128, 16, 2, nb)
+    assert e.value.status == -9 and "cudaMalloc" in str(e.value)
+    p = wk.Pool(2, 2, 64, 16, 2, 4)
+    assert p.nbytes == 2 * 2 * 4 * 2 * 16 * 64 * 2
+    torch.cuda.synchronize()
