@@ -25,9 +25,15 @@
  *   - Ops are asynchronous on the given stream, never allocate and never synchronise the
  *     host; they are CUDA-graph capturable.  Asynchronous CUDA faults surface at
  *     the caller's next synchronisation, as with any CUDA call.
- *   - Each kernel op uses one of 512 per-device arrival-counter slots (round robin): at
- *     most 512 ops may EXECUTE concurrently on one device across streams (any number may
- *     be queued on one stream, where ops run in order).
+ *   - Each kernel op owns one per-device arrival-counter slot from enqueue until it has
+ *     finished with it (its last layer published).  An op takes its stream's previous slot
+ *     (ops on one stream run in order, so any number may be queued on one stream), else a
+ *     slot whose op is done: ops of at most 512 STREAMS may be pending on one device at
+ *     once; an op on a 513th stream fails with WIND_ERR_UNSUPPORTED, nothing enqueued.  A
+ *     pending op (e.g. a stepped migration waiting on decode steps) keeps its slot however
+ *     many ops other streams run meanwhile.  Ops captured into a CUDA graph take one of
+ *     512 separate graph slots round robin: at most 512 captured ops may execute
+ *     concurrently on one device.
  *   - `cudaStream_t` parameters are passed as `void*` (0 = the legacy default stream) so
  *     the header needs no CUDA include.
  *   - The copy kernels use programmatic dependent launch: each waits for the previous

@@ -17,6 +17,7 @@
 #include <atomic>
 #include <mutex>
 #include <string>
+#include <unordered_map>
 #include <vector>
 
 #include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: ranges show up in ncu / nsys, free otherwise
@@ -90,11 +91,23 @@ struct DevCtx {
   uint8_t uuid[16] = {};
   uint32_t* counters = nullptr;  // kCounterSlots * WIND_KV_MAX_LAYERS, zeroed
   unsigned long long* stamps = nullptr;  // kCounterSlots: start time of a burst-paced op
-  std::atomic<uint64_t> seq{0};
+  uint32_t* op_layers = nullptr;  // kCounterSlots: layers an op has published (device)
+  // Eager slot ownership (take_slot): slot s is free when done_host[s] == assigned[s]; the
+  // GPU writes done_host (mapped pinned memory) when the slot's op has finished with it.
+  std::mutex slot_mu;
+  uint32_t* done_host = nullptr;  // kEagerSlots
+  uint32_t assigned[kEagerSlots] = {};
+  unsigned long long owner[kEagerSlots] = {};  // stream id of the slot's last op (0: unknown)
+  std::unordered_map<unsigned long long, int> slot_of_stream;
+  uint32_t next_seq = 0;
+  int cursor = 0;
+  std::atomic<uint64_t> graph_seq{0};
   size_t tma_smem_set = 0;
   int32_t* err = nullptr;        // debug device-check word
-  uint32_t* scratch = nullptr;   // debug table-check scratch
-  int32_t scratch_n = 0;
+  // debug table-check scratch, per counter slot: the op owning the slot is its only user
+  // (two debug ops on different streams never share one)
+  uint32_t* scratch[kCounterSlots] = {};
+  int32_t scratch_n[kCounterSlots] = {};
 };
 
 constexpr int kMaxDevices = 64;
@@ -119,6 +132,11 @@ wind_status dev_ctx(int dev, DevCtx** out) {
     WKV_CUDA(cudaMalloc(&c.counters, cbytes), "cudaMalloc(counters)");
     WKV_CUDA(cudaMemset(c.counters, 0, cbytes), "cudaMemset(counters)");
     WKV_CUDA(cudaMalloc(&c.stamps, sizeof(unsigned long long) * kCounterSlots), "cudaMalloc(stamps)");
+    WKV_CUDA(cudaMalloc(&c.op_layers, sizeof(uint32_t) * kCounterSlots), "cudaMalloc(op_layers)");
+    WKV_CUDA(cudaMemset(c.op_layers, 0, sizeof(uint32_t) * kCounterSlots), "cudaMemset(op_layers)");
+    WKV_CUDA(cudaHostAlloc(&c.done_host, sizeof(uint32_t) * kEagerSlots,
+                           cudaHostAllocMapped | cudaHostAllocPortable), "cudaHostAlloc(slot done words)");
+    memset(c.done_host, 0, sizeof(uint32_t) * kEagerSlots);
     WKV_CUDA(cudaMalloc(&c.err, sizeof(int32_t)), "cudaMalloc(err)");
     WKV_CUDA(cudaMemset(c.err, 0, sizeof(int32_t)), "cudaMemset(err)");
     const size_t max_smem = 227 * 1024;
@@ -784,22 +802,20 @@ struct OpItem {
 };
 
 // Debug pools: device-side table check (not on the release hot path; may allocate scratch).
-wind_status debug_check(DevCtx* ctx, int exec, const wind_kv_pool* src, const OpItem& it,
+// Runs in the op's stream with the scratch of the op's counter slot.
+wind_status debug_check(DevCtx* ctx, int exec, int slot, const wind_kv_pool* src, const OpItem& it,
                         cudaStream_t s) {
   const int32_t need = std::max(src->desc.n_blocks, it.dst->desc.n_blocks);
-  if (ctx->scratch_n < need) {
-    std::lock_guard<std::mutex> lk(ctx->mu);
-    if (ctx->scratch_n < need) {
-      DeviceGuard g(exec);
-      if (ctx->scratch) cudaFree(ctx->scratch);
-      ctx->scratch = nullptr;
-      ctx->scratch_n = 0;
-      WKV_CUDA(cudaMalloc(&ctx->scratch, sizeof(uint32_t) * 2 * need), "cudaMalloc(debug scratch)");
-      ctx->scratch_n = need;
-    }
+  if (ctx->scratch_n[slot] < need) {
+    DeviceGuard g(exec);
+    if (ctx->scratch[slot]) cudaFree(ctx->scratch[slot]);  // synchronises: no launch still uses it
+    ctx->scratch[slot] = nullptr;
+    ctx->scratch_n[slot] = 0;
+    WKV_CUDA(cudaMalloc(&ctx->scratch[slot], sizeof(uint32_t) * 2 * need), "cudaMalloc(debug scratch)");
+    ctx->scratch_n[slot] = need;
   }
   WKV_CUDA(launch_table_check(it.sbt, it.dbt, it.n, src->desc.n_blocks, it.dst->desc.n_blocks,
-                              src->base == it.dst->base, ctx->scratch, ctx->scratch_n, ctx->err, s),
+                              src->base == it.dst->base, ctx->scratch[slot], ctx->scratch_n[slot], ctx->err, s),
            "table check launch");
   g_launches += 2;
   return WIND_OK;
@@ -821,17 +837,9 @@ bool host_readable(const void* ptr) {
 // each pool's plane stride).  The tables must be host-readable (the driver needs every
 // address at enqueue time); the layer flags are published by one tiny kernel afterwards
 // (stream order: after every copy), so per-layer streaming is not available on this path.
-wind_status copy_engine_op(const Params& p, int32_t src_nb, const OpItem* items, int n_items,
-                           cudaStream_t s, int32_t rate_mbps) {
-  const size_t rows = static_cast<size_t>(2) * p.n_layers;
-  // rate limit: a pace kernel stamps the op start; after copies worth >= 20 us of the
-  // budget, a pace kernel holds the stream until start + bytes_so_far / rate.  The stamp
-  // lives in this op's (otherwise unused) arrival-counter slot.
-  unsigned long long* t0 = reinterpret_cast<unsigned long long*>(p.counters + WIND_KV_MAX_LAYERS - 2);
-  double sched_ns = 0, last_paced = 0;
-  int launches = 0;
-  // the tables are read here, on the CPU: check them before anything is enqueued (an entry
-  // out of range would make a DMA copy write outside both pools)
+// The copy-engine path reads the tables on the CPU: check them before anything is enqueued
+// (an entry out of range would make a DMA copy write outside both pools).
+wind_status check_ce_tables(int32_t src_nb, const OpItem* items, int n_items) {
   for (int j = 0; j < n_items; ++j) {
     const OpItem& it = items[j];
     if (it.n == 0) continue;
@@ -843,6 +851,86 @@ wind_status copy_engine_op(const Params& p, int32_t src_nb, const OpItem* items,
         return fail(WIND_ERR_BLOCK_RANGE, "item %d: table entry %d out of range (src %d of %d, dst %d of %d)",
                     j, i, it.sbt[i], src_nb, it.dbt[i], it.dst->desc.n_blocks);
   }
+  return WIND_OK;
+}
+
+// Counter-slot ownership (wind_kv_internal.h kEagerSlots).  An eager op takes the slot its
+// stream's previous op used if that slot is still that stream's (stream order keeps the two
+// apart), else the next slot whose last op has marked it done (done_host == assigned).
+// Nothing is enqueued here; release_slot undoes a take when the op fails before launching.
+struct Slot {
+  int index = -1;
+  uint32_t seq = 0;       // 0: not tracked (captured op)
+  uint32_t prev_assigned = 0;
+  unsigned long long prev_owner = 0;
+};
+
+wind_status take_slot(DevCtx* ctx, int exec, cudaStream_t s, Slot* out) {
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  if (cudaStreamIsCapturing(s, &cap) != cudaSuccess) {
+    cudaGetLastError();
+    cap = cudaStreamCaptureStatusNone;
+  }
+  if (cap != cudaStreamCaptureStatusNone) {  // a graph replay cannot report back: round robin
+    out->index = kEagerSlots + static_cast<int>(ctx->graph_seq.fetch_add(1) % kGraphSlots);
+    out->seq = 0;
+    return WIND_OK;
+  }
+  unsigned long long sid = 0;
+  if (cudaStreamGetId(s, &sid) != cudaSuccess) {
+    cudaGetLastError();
+    sid = 0;
+  }
+  std::lock_guard<std::mutex> lk(ctx->slot_mu);
+  int idx = -1;
+  if (sid) {
+    auto it = ctx->slot_of_stream.find(sid);
+    if (it != ctx->slot_of_stream.end() && ctx->owner[it->second] == sid) idx = it->second;
+  }
+  for (int probe = 0; idx < 0 && probe < kEagerSlots; ++probe) {
+    const int i = (ctx->cursor + probe) % kEagerSlots;
+    if (*reinterpret_cast<volatile uint32_t*>(ctx->done_host + i) == ctx->assigned[i]) {
+      idx = i;
+      ctx->cursor = (i + 1) % kEagerSlots;
+    }
+  }
+  if (idx < 0)
+    return fail(WIND_ERR_UNSUPPORTED, "ops of %d streams are in flight on device %d (the counter-slot "
+                "limit); nothing enqueued", kEagerSlots, exec);
+  uint32_t seq = ++ctx->next_seq;
+  if (seq == 0) seq = ++ctx->next_seq;  // 0 is the initial done word
+  out->index = idx;
+  out->seq = seq;
+  out->prev_assigned = ctx->assigned[idx];
+  out->prev_owner = ctx->owner[idx];
+  if (ctx->owner[idx] && ctx->owner[idx] != sid) ctx->slot_of_stream.erase(ctx->owner[idx]);
+  ctx->assigned[idx] = seq;
+  ctx->owner[idx] = sid;
+  if (sid) ctx->slot_of_stream[sid] = idx;
+  return WIND_OK;
+}
+
+void release_slot(DevCtx* ctx, const Slot& sl) {
+  if (sl.seq == 0 || sl.index < 0) return;
+  std::lock_guard<std::mutex> lk(ctx->slot_mu);
+  if (ctx->assigned[sl.index] != sl.seq) return;
+  const unsigned long long sid = ctx->owner[sl.index];
+  ctx->assigned[sl.index] = sl.prev_assigned;
+  ctx->owner[sl.index] = sl.prev_owner;
+  if (sid && sid != sl.prev_owner) ctx->slot_of_stream.erase(sid);
+  if (sl.prev_owner) ctx->slot_of_stream[sl.prev_owner] = sl.index;
+}
+
+wind_status copy_engine_op(const Params& p, int32_t src_nb, const OpItem* items, int n_items,
+                           cudaStream_t s, int32_t rate_mbps) {
+  const size_t rows = static_cast<size_t>(2) * p.n_layers;
+  // rate limit: a pace kernel stamps the op start; after copies worth >= 20 us of the
+  // budget, a pace kernel holds the stream until start + bytes_so_far / rate.  The stamp
+  // lives in this op's (otherwise unused) arrival-counter slot.
+  unsigned long long* t0 = reinterpret_cast<unsigned long long*>(p.counters + WIND_KV_MAX_LAYERS - 2);
+  double sched_ns = 0, last_paced = 0;
+  int launches = 0;
+  (void)src_nb;  // the tables were range-checked by check_ce_tables before the slot was taken
   if (rate_mbps > 0) {
     WKV_CUDA(launch_pace(t0, 0, 1, s), "pace kernel launch");
     ++launches;
@@ -1130,12 +1218,9 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     if (path == WIND_PATH_HOST || dbg || t.kernel == kCopyEngine || t.kernel == kStaged)
       return fail(WIND_ERR_UNSUPPORTED, "step-aligned ops need device pools, an SM kernel and no debug pool");
   }
-  bool debug = false;
+  bool debug = false;  // the device-side table check is enqueued once the op's slot is taken
   for (int j = 0; j < n_items; ++j)
-    if (items[j].n > 0 && ((src->desc.flags | items[j].dst->desc.flags) & WIND_POOL_DEBUG)) {
-      if ((st = debug_check(ctx, exec, src, items[j], s)) != WIND_OK) return st;
-      debug = true;
-    }
+    debug = debug || (items[j].n > 0 && ((src->desc.flags | items[j].dst->desc.flags) & WIND_POOL_DEBUG));
 
   // HOST path: the staged copy-engine path only when the caller asks for it (kernel 4, via
   // wind_kv_set_tuning or a per-op wind_kv_migrate_ex override).  It reads the host-side
@@ -1228,9 +1313,23 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   p.n_items = ni;
   p.units_per_plane = base_units;
   p.total_units = static_cast<int64_t>(2) * p.n_layers * base_units;
-  const uint64_t slot = ctx->seq.fetch_add(1) % kCounterSlots;
-  p.counters = ctx->counters + slot * WIND_KV_MAX_LAYERS;
+  if (kernel == kCopyEngine && (st = check_ce_tables(src->desc.n_blocks, items, n_items)) != WIND_OK) return st;
+  // the op's counter slot: the last step that may fail without enqueuing anything
+  Slot sl;
+  if ((st = take_slot(ctx, exec, s, &sl)) != WIND_OK) return st;
+  const int slot = sl.index;
+  p.counters = ctx->counters + static_cast<size_t>(slot) * WIND_KV_MAX_LAYERS;
+  p.op_layers = ctx->op_layers + slot;
+  p.done_word = sl.seq ? ctx->done_host + slot : nullptr;
+  p.op_seq = sl.seq;
   p.abort_word = debug ? ctx->err : nullptr;
+  if (debug)
+    for (int j = 0; j < n_items; ++j)
+      if (items[j].n > 0 && ((src->desc.flags | items[j].dst->desc.flags) & WIND_POOL_DEBUG))
+        if ((st = debug_check(ctx, exec, slot, src, items[j], s)) != WIND_OK) {
+          release_slot(ctx, sl);
+          return st;
+        }
 
   p.fan = fan;
   if (fan > 1) {  // every item walks items[0]'s units
@@ -1298,6 +1397,10 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     slice_units = std::max<int64_t>(slice_units, grid);  // a burst keeps the whole grid busy
     unsigned long long* t0 = ctx->stamps + slot;
     p.ns_per_byte = 0.f;
+    // a burst-paced op's last pace kernel (after every slice, in stream order) frees the
+    // slot; a stepped op's last layer publication does (op_layer_published)
+    uint32_t* const done_word = p.done_word;
+    if (!step) p.done_word = nullptr;
     static PFN_waitValue32 wait_fn = driver_fn<PFN_waitValue32>("cuStreamWaitValue32");
     if (step && !wait_fn) return fail(WIND_ERR_CUDA, "cuStreamWaitValue32 entry point unavailable");
     int launches = 0;
@@ -1323,7 +1426,9 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
       // hold the stream until the schedule reaches the bytes moved so far (after the last
       // slice too: the op then ends when its rate says, as the in-kernel pacer's ops do)
       const double done = payload * static_cast<double>(p.unit_hi) / static_cast<double>(p.total_units);
-      WKV_CUDA(launch_pace(t0, static_cast<uint64_t>(done * 1e3 / t.rate_mbps), 0, s), "pace kernel launch");
+      const bool last = p.unit_hi == p.total_units;
+      WKV_CUDA(launch_pace(t0, static_cast<uint64_t>(done * 1e3 / t.rate_mbps), 0, s,
+                           last ? done_word : nullptr, p.op_seq), "pace kernel launch");
       ++launches;
     }
     g_launches += launches;

@@ -191,10 +191,12 @@ def test_plain_c_abi_user():
 
 
 def test_many_concurrent_ops_across_streams():
-    """200 ops enqueued at once on 200 streams (each into its own destination pool), plus
-    a 40-op layer-streamed sequence on one stream: every op takes its own arrival-counter
-    slot; all data byte-exact vs the oracle, every flag == its ticket."""
+    """200 ops enqueued at once on 200 distinct CUDA streams (each into its own destination
+    pool), plus a 40-op layer-streamed sequence on one stream: every pending op holds its
+    own arrival-counter slot; all data byte-exact vs the oracle, every flag == its ticket."""
     import oracle as O
+    from rawstreams import raw_streams
+    raws = raw_streams(200)
     L, H, d, bs, eb = 4, 2, 64, 16, 2
     rng = np.random.default_rng(7)
     src = wk.Pool(L, H, d, bs, eb, 64)
@@ -207,7 +209,7 @@ def test_many_concurrent_ops_across_streams():
         sbt = rng.permutation(64)[:20].astype(np.int32)
         dbt = rng.permutation(32)[:20].astype(np.int32)
         dsts.append(p)
-        jobs.append((p, torch.cuda.Stream(), torch.as_tensor(sbt, device="cuda"),
+        jobs.append((p, raws[k].handle, torch.as_tensor(sbt, device="cuda"),
                      torch.as_tensor(dbt, device="cuda"), sbt, dbt))
     torch.cuda.synchronize()
     for p, st, ts, td, _, _ in jobs:
@@ -228,6 +230,8 @@ def test_many_concurrent_ops_across_streams():
         np.testing.assert_array_equal(p.tensor().cpu().numpy(), want)
         assert [p.layer_count(l) for l in range(L)] == [1] * L
     assert one.layer_ticket() == 40 and [one.layer_count(l) for l in range(L)] == [40] * L
+    for r in raws:
+        r.destroy()
 
 
 def test_ops_enqueued_from_many_host_threads():

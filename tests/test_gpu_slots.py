@@ -1,0 +1,226 @@
+"""GPU: ownership of the per-op arrival-counter slots (include/wind_kv.h "Conventions";
+wind_kv_internal.h kEagerSlots).
+
+An op counts its CTAs' arrivals per layer in a counter slot and publishes a layer when the
+count completes (A5).  A slot must never be shared by two ops that execute at the
+same time.  Round 1-2 handed slots out round robin at enqueue, so an op that stayed pending
+for long — a stepped migration waiting on decode steps, an op queued behind a
+layer_wait — had its slot handed to the 512th op enqueued after it on another stream.
+These tests hold such an op pending while hundreds of ops run elsewhere, and fill every
+slot with pending ops, then compare every byte and flag with the oracle.
+
+The gates are host-mapped words (a host pool's layer flags) released by a CPU store, with
+a watchdog thread that releases them anyway: a blocked stream can never hang the suite."""
+import ctypes as ct
+import threading
+import time
+
+import numpy as np
+import pytest
+import torch
+
+import oracle as O
+import paper_conf_isca_fenghzly025_b200 as wk
+from rawstreams import raw_streams
+
+pytestmark = pytest.mark.gpu
+DEV = torch.device("cuda", 0)
+
+
+class HostGate:
+    """A uint32 in mapped pinned memory (layer 0 flag of a 1-layer host pool): streams wait
+    on it on the GPU (cuStreamWaitValue32), the CPU releases them with a plain store."""
+
+    def __init__(self, watchdog_s: float):
+        self.pool = wk.Pool(1, 1, 64, 16, 2, 1, loc="host")
+        self.word = ct.c_uint32.from_address(self.pool.flags_ptr)
+        self.word.value = 0
+        self._stop = threading.Event()
+        self._th = threading.Thread(target=self._watch, args=(watchdog_s,), daemon=True)
+        self._th.start()
+
+    def _watch(self, s):
+        if not self._stop.wait(s):
+            self.word.value = 1 << 20  # the test hung: release every waiter
+
+    def set(self, v: int) -> None:
+        self.word.value = v
+
+    def close(self) -> None:
+        self.word.value = 1 << 20
+        self._stop.set()
+
+
+def geom(L, H, d, bs, eb, nb):
+    return O.Geom(0, L, H, d, bs, eb, nb)
+
+
+def test_pending_stepped_op_keeps_its_counter_slot():
+    """A stepped op (slices released by a host-driven step counter) runs its first slice and
+    then waits; meanwhile 700 ops over the same layers run to completion on another stream.
+    The stepped op keeps its slot: after its remaining slices both destinations equal the
+    oracle and every flag counts its ops (1 and 700)."""
+    L, H, d, bs, eb = 6, 8, 128, 16, 2  # 32 KiB chunks
+    nb, n = 64, 48
+    rng = np.random.default_rng(31)
+    src = wk.Pool(L, H, d, bs, eb, nb)
+    dst = wk.Pool(L, H, d, bs, eb, nb)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    d0 = rng.integers(0, 256, dst.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    dst.tensor().copy_(torch.from_numpy(d0))
+    sbt = rng.permutation(nb)[:n].astype(np.int32)
+    dbt = rng.permutation(nb)[:n].astype(np.int32)
+    ts, td = torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)
+    osrc = wk.Pool(L, H, d, bs, eb, 16)
+    odst = wk.Pool(L, H, d, bs, eb, 16)
+    o0 = rng.integers(0, 256, osrc.nbytes, dtype=np.uint8)
+    osrc.tensor().copy_(torch.from_numpy(o0))
+    odst.tensor().zero_()
+    obt_s = np.array([3, 9, 1, 14], np.int32)
+    obt_d = np.array([0, 5, 6, 11], np.int32)
+    tos, tod = torch.as_tensor(obt_s, device=DEV), torch.as_tensor(obt_d, device=DEV)
+    mig, other = torch.cuda.Stream(DEV), torch.cuda.Stream(DEV)
+    torch.cuda.synchronize()
+    gate = HostGate(watchdog_s=60)
+    try:
+        n0 = wk.launch_count()
+        payload = 2 * L * n * src.chunk_bytes
+        wk.migrate_stepped(src, ts, dst, td, gate.pool.flags_ptr, first_step=1,
+                           bytes_per_step=payload // 4 + 1, stream=mig)
+        slices = wk.launch_count() - n0
+        assert slices >= 4
+        gate.set(1)  # slice 0 runs, the rest wait for steps 2, 3, ...
+        time.sleep(0.05)
+        for _ in range(700):
+            wk.migrate(osrc, tos, odst, tod, stream=other)
+        other.synchronize()
+        assert not mig.query(), "the stepped op should still be waiting for step 2"
+        gate.set(slices)
+        mig.synchronize()
+    finally:
+        gate.close()
+        torch.cuda.synchronize()
+    want = d0.copy()
+    assert O.migrate(s0, geom(L, H, d, bs, eb, nb), sbt, want, geom(L, H, d, bs, eb, nb), dbt, 0, L) == O.OK
+    np.testing.assert_array_equal(dst.tensor().cpu().numpy(), want)
+    assert [dst.layer_count(l) for l in range(L)] == [1] * L
+    owant = np.zeros(odst.nbytes, np.uint8)
+    assert O.migrate(o0, geom(L, H, d, bs, eb, 16), obt_s, owant, geom(L, H, d, bs, eb, 16), obt_d, 0, L) == O.OK
+    np.testing.assert_array_equal(odst.tensor().cpu().numpy(), owant)
+    assert [odst.layer_count(l) for l in range(L)] == [700] * L
+
+
+def test_counter_slots_exhaust_cleanly_and_recover():
+    """512 streams each hold a pending op (queued behind a host gate): an op on a 513th
+    stream is UNSUPPORTED with nothing enqueued, while a held stream may still queue more
+    (its ops share its slot in stream order).  After the gate opens every destination
+    equals the oracle and the 513th stream's op goes through."""
+    L, H, d, bs, eb = 2, 1, 64, 16, 2  # 2 KiB chunks
+    rng = np.random.default_rng(32)
+    src = wk.Pool(L, H, d, bs, eb, 8)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    k = 512
+    dsts = [wk.Pool(L, H, d, bs, eb, 8) for _ in range(k + 1)]
+    for p in dsts:
+        p.tensor().zero_()
+    sbt = np.array([7, 2, 5, 0], np.int32)
+    dbt = np.array([1, 3, 4, 6], np.int32)
+    ts, td = torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)
+    streams = raw_streams(k + 1)  # distinct CUDA streams (torch recycles 32)
+    torch.cuda.synchronize()  # every earlier op of the session is done: all slots free
+    gate = HostGate(watchdog_s=90)
+    try:
+        for i in range(k):
+            wk.layer_wait(gate.pool, 0, 1, stream=streams[i].handle)
+            wk.migrate(src, ts, dsts[i], td, stream=streams[i].handle)
+        n0 = wk.launch_count()
+        with pytest.raises(wk.WindKVError) as e:
+            wk.migrate(src, ts, dsts[k], td, stream=streams[k].handle)
+        assert e.value.status == -10 and "counter-slot" in wk.last_error()
+        assert wk.launch_count() == n0 and dsts[k].layer_ticket() == 0
+        wk.migrate(src, ts, dsts[0], td, layer_lo=1, layer_hi=2, stream=streams[0].handle)  # same stream: OK
+        gate.set(1)
+        for st in streams[:k]:
+            st.synchronize()
+    finally:
+        gate.close()
+        torch.cuda.synchronize()
+    wk.migrate(src, ts, dsts[k], td, stream=streams[k].handle)  # slots are free again
+    torch.cuda.synchronize()
+    for st in streams:
+        st.destroy()
+    want = np.zeros(src.nbytes, np.uint8)
+    g = geom(L, H, d, bs, eb, 8)
+    assert O.migrate(s0, g, sbt, want, g, dbt, 0, L) == O.OK
+    for i, p in enumerate(dsts):
+        np.testing.assert_array_equal(p.tensor().cpu().numpy(), want)
+        assert [p.layer_count(l) for l in range(L)] == ([2, 2] if i == 0 else [1, 1])
+
+
+def test_captured_ops_use_their_own_slots_and_replay_while_eager_ops_run():
+    """A captured op (graph slot ring) replayed on one stream while eager ops run on
+    another: both destinations equal the oracle, flags count every replay and op."""
+    L, H, d, bs, eb = 4, 2, 64, 16, 2
+    rng = np.random.default_rng(33)
+    src = wk.Pool(L, H, d, bs, eb, 32)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    a, b = wk.Pool(L, H, d, bs, eb, 32), wk.Pool(L, H, d, bs, eb, 32)
+    a.tensor().zero_()
+    b.tensor().zero_()
+    sbt = rng.permutation(32)[:20].astype(np.int32)
+    dbt = rng.permutation(32)[:20].astype(np.int32)
+    ts, td = torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)
+    cap, eager = torch.cuda.Stream(DEV), torch.cuda.Stream(DEV)
+    torch.cuda.synchronize()
+    graph = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(graph, stream=cap):
+        wk.migrate(src, ts, a, td, stream=cap)
+    torch.cuda.synchronize()
+    for _ in range(50):
+        with torch.cuda.stream(cap):
+            graph.replay()
+        wk.migrate(src, ts, b, td, stream=eager)
+    torch.cuda.synchronize()
+    want = np.zeros(src.nbytes, np.uint8)
+    g = geom(L, H, d, bs, eb, 32)
+    assert O.migrate(s0, g, sbt, want, g, dbt, 0, L) == O.OK
+    for p in (a, b):
+        np.testing.assert_array_equal(p.tensor().cpu().numpy(), want)
+        assert [p.layer_count(l) for l in range(L)] == [50] * L
+
+
+def test_debug_table_checks_on_two_streams_do_not_share_scratch():
+    """Debug pools run a device-side table check (count kernel + judge kernel over a scratch
+    array) before the copy.  Two valid debug ops on two streams at the same time use the
+    scratch of their own counter slots: no false DUP_DST / ALIAS, and both copies land."""
+    L, H, d, bs, eb = 1, 1, 8, 16, 2  # 256-byte chunks: the table check dominates
+    nb, n = 200_000, 150_000
+    rng = np.random.default_rng(34)
+    src = wk.Pool(L, H, d, bs, eb, nb, debug=True)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    dsts = [wk.Pool(L, H, d, bs, eb, nb, debug=True) for _ in range(2)]
+    for p in dsts:
+        p.tensor().zero_()
+    tabs = []
+    for _ in range(2):
+        sbt = rng.permutation(nb)[:n].astype(np.int32)
+        dbt = rng.permutation(nb)[:n].astype(np.int32)
+        tabs.append((sbt, dbt, torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)))
+    streams = [torch.cuda.Stream(DEV) for _ in range(2)]
+    torch.cuda.synchronize()
+    for _ in range(10):
+        for p, (_, _, ts, td), st in zip(dsts, tabs, streams):
+            wk.migrate(src, ts, p, td, stream=st)
+    torch.cuda.synchronize()
+    for p in dsts:
+        wk.check_device_error(p)  # raises DEVICE_CHECK on a (false) table error
+    g = geom(L, H, d, bs, eb, nb)
+    for p, (sbt, dbt, _, _) in zip(dsts, tabs):
+        want = np.zeros(p.nbytes, np.uint8)
+        assert O.migrate(s0, g, sbt, want, g, dbt, 0, L) == O.OK
+        np.testing.assert_array_equal(p.tensor().cpu().numpy(), want)
+        assert p.layer_count(0) == 10
