@@ -26,7 +26,7 @@
  *     host; they are CUDA-graph capturable.  Asynchronous CUDA faults surface at
  *     the caller's next synchronisation, as with any CUDA call.
  *   - Each kernel op owns one per-device arrival-counter slot from enqueue until it has
- *     finished with it (its last layer published).  An op takes its stream's previous slot
+ *     completed (a host-side event recorded after it).  An op takes its stream's previous slot
  *     (ops on one stream run in order, so any number may be queued on one stream), else a
  *     slot whose op is done: ops of at most 512 STREAMS may be pending on one device at
  *     once; an op on a 513th stream fails with WIND_ERR_UNSUPPORTED, nothing enqueued.  A

@@ -91,15 +91,13 @@ struct DevCtx {
   uint8_t uuid[16] = {};
   uint32_t* counters = nullptr;  // kCounterSlots * WIND_KV_MAX_LAYERS, zeroed
   unsigned long long* stamps = nullptr;  // kCounterSlots: start time of a burst-paced op
-  uint32_t* op_layers = nullptr;  // kCounterSlots: layers an op has published (device)
-  // Eager slot ownership (take_slot): slot s is free when done_host[s] == assigned[s]; the
-  // GPU writes done_host (mapped pinned memory) when the slot's op has finished with it.
+  // Eager slot ownership (take_slot): after every eager op, done[s] is recorded on the op's
+  // stream; slot s is free for another stream once done[s] has completed.
   std::mutex slot_mu;
-  uint32_t* done_host = nullptr;  // kEagerSlots
-  uint32_t assigned[kEagerSlots] = {};
+  cudaEvent_t done[kEagerSlots] = {};
+  bool used[kEagerSlots] = {};
   unsigned long long owner[kEagerSlots] = {};  // stream id of the slot's last op (0: unknown)
   std::unordered_map<unsigned long long, int> slot_of_stream;
-  uint32_t next_seq = 0;
   int cursor = 0;
   std::atomic<uint64_t> graph_seq{0};
   size_t tma_smem_set = 0;
@@ -132,11 +130,8 @@ wind_status dev_ctx(int dev, DevCtx** out) {
     WKV_CUDA(cudaMalloc(&c.counters, cbytes), "cudaMalloc(counters)");
     WKV_CUDA(cudaMemset(c.counters, 0, cbytes), "cudaMemset(counters)");
     WKV_CUDA(cudaMalloc(&c.stamps, sizeof(unsigned long long) * kCounterSlots), "cudaMalloc(stamps)");
-    WKV_CUDA(cudaMalloc(&c.op_layers, sizeof(uint32_t) * kCounterSlots), "cudaMalloc(op_layers)");
-    WKV_CUDA(cudaMemset(c.op_layers, 0, sizeof(uint32_t) * kCounterSlots), "cudaMemset(op_layers)");
-    WKV_CUDA(cudaHostAlloc(&c.done_host, sizeof(uint32_t) * kEagerSlots,
-                           cudaHostAllocMapped | cudaHostAllocPortable), "cudaHostAlloc(slot done words)");
-    memset(c.done_host, 0, sizeof(uint32_t) * kEagerSlots);
+    for (int i = 0; i < kEagerSlots; ++i)
+      WKV_CUDA(cudaEventCreateWithFlags(&c.done[i], cudaEventDisableTiming), "cudaEventCreate(slot)");
     WKV_CUDA(cudaMalloc(&c.err, sizeof(int32_t)), "cudaMalloc(err)");
     WKV_CUDA(cudaMemset(c.err, 0, sizeof(int32_t)), "cudaMemset(err)");
     const size_t max_smem = 227 * 1024;
@@ -856,13 +851,14 @@ wind_status check_ce_tables(int32_t src_nb, const OpItem* items, int n_items) {
 
 // Counter-slot ownership (wind_kv_internal.h kEagerSlots).  An eager op takes the slot its
 // stream's previous op used if that slot is still that stream's (stream order keeps the two
-// apart), else the next slot whose last op has marked it done (done_host == assigned).
-// Nothing is enqueued here; release_slot undoes a take when the op fails before launching.
+// apart), else a slot whose last op has completed (its done event).  No device work: the
+// event is recorded after the op's launches (finish_slot).  Nothing is enqueued here;
+// release_slot undoes a take when the op fails before launching.
 struct Slot {
   int index = -1;
-  uint32_t seq = 0;       // 0: not tracked (captured op)
-  uint32_t prev_assigned = 0;
-  unsigned long long prev_owner = 0;
+  bool eager = false;
+  bool prev_used = false;
+  unsigned long long sid = 0, prev_owner = 0;
 };
 
 wind_status take_slot(DevCtx* ctx, int exec, cudaStream_t s, Slot* out) {
@@ -871,9 +867,9 @@ wind_status take_slot(DevCtx* ctx, int exec, cudaStream_t s, Slot* out) {
     cudaGetLastError();
     cap = cudaStreamCaptureStatusNone;
   }
-  if (cap != cudaStreamCaptureStatusNone) {  // a graph replay cannot report back: round robin
+  if (cap != cudaStreamCaptureStatusNone) {  // a replay cannot be tracked here: round robin
     out->index = kEagerSlots + static_cast<int>(ctx->graph_seq.fetch_add(1) % kGraphSlots);
-    out->seq = 0;
+    out->eager = false;
     return WIND_OK;
   }
   unsigned long long sid = 0;
@@ -889,35 +885,44 @@ wind_status take_slot(DevCtx* ctx, int exec, cudaStream_t s, Slot* out) {
   }
   for (int probe = 0; idx < 0 && probe < kEagerSlots; ++probe) {
     const int i = (ctx->cursor + probe) % kEagerSlots;
-    if (*reinterpret_cast<volatile uint32_t*>(ctx->done_host + i) == ctx->assigned[i]) {
+    if (!ctx->used[i]) {
       idx = i;
-      ctx->cursor = (i + 1) % kEagerSlots;
+    } else {
+      const cudaError_t q = cudaEventQuery(ctx->done[i]);
+      if (q == cudaSuccess) idx = i;
+      else if (q != cudaErrorNotReady) cudaGetLastError();
     }
+    if (idx >= 0) ctx->cursor = (i + 1) % kEagerSlots;
   }
   if (idx < 0)
     return fail(WIND_ERR_UNSUPPORTED, "ops of %d streams are in flight on device %d (the counter-slot "
                 "limit); nothing enqueued", kEagerSlots, exec);
-  uint32_t seq = ++ctx->next_seq;
-  if (seq == 0) seq = ++ctx->next_seq;  // 0 is the initial done word
   out->index = idx;
-  out->seq = seq;
-  out->prev_assigned = ctx->assigned[idx];
+  out->eager = true;
+  out->sid = sid;
+  out->prev_used = ctx->used[idx];
   out->prev_owner = ctx->owner[idx];
   if (ctx->owner[idx] && ctx->owner[idx] != sid) ctx->slot_of_stream.erase(ctx->owner[idx]);
-  ctx->assigned[idx] = seq;
+  ctx->used[idx] = true;
   ctx->owner[idx] = sid;
   if (sid) ctx->slot_of_stream[sid] = idx;
   return WIND_OK;
 }
 
+// After the op's last launch: its slot is busy until the stream gets past this point.
+wind_status finish_slot(DevCtx* ctx, const Slot& sl, cudaStream_t s) {
+  if (!sl.eager) return WIND_OK;
+  WKV_CUDA(cudaEventRecord(ctx->done[sl.index], s), "cudaEventRecord(slot)");
+  return WIND_OK;
+}
+
 void release_slot(DevCtx* ctx, const Slot& sl) {
-  if (sl.seq == 0 || sl.index < 0) return;
+  if (!sl.eager) return;
   std::lock_guard<std::mutex> lk(ctx->slot_mu);
-  if (ctx->assigned[sl.index] != sl.seq) return;
-  const unsigned long long sid = ctx->owner[sl.index];
-  ctx->assigned[sl.index] = sl.prev_assigned;
+  if (ctx->owner[sl.index] != sl.sid) return;
+  if (sl.sid && sl.sid != sl.prev_owner) ctx->slot_of_stream.erase(sl.sid);
+  ctx->used[sl.index] = sl.prev_used;
   ctx->owner[sl.index] = sl.prev_owner;
-  if (sid && sid != sl.prev_owner) ctx->slot_of_stream.erase(sid);
   if (sl.prev_owner) ctx->slot_of_stream[sl.prev_owner] = sl.index;
 }
 
@@ -1319,9 +1324,6 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   if ((st = take_slot(ctx, exec, s, &sl)) != WIND_OK) return st;
   const int slot = sl.index;
   p.counters = ctx->counters + static_cast<size_t>(slot) * WIND_KV_MAX_LAYERS;
-  p.op_layers = ctx->op_layers + slot;
-  p.done_word = sl.seq ? ctx->done_host + slot : nullptr;
-  p.op_seq = sl.seq;
   p.abort_word = debug ? ctx->err : nullptr;
   if (debug)
     for (int j = 0; j < n_items; ++j)
@@ -1341,7 +1343,10 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     p.total_units = static_cast<int64_t>(2) * p.n_layers * p.units_per_plane;
   }
   if (kernel == kCopyEngine) {
-    if ((st = copy_engine_op(p, src->desc.n_blocks, items, n_items, s, t.rate_mbps)) != WIND_OK) return st;
+    st = copy_engine_op(p, src->desc.n_blocks, items, n_items, s, t.rate_mbps);
+    const wind_status fs = finish_slot(ctx, sl, s);  // whatever was enqueued holds the slot
+    if (st != WIND_OK) return st;
+    if (fs != WIND_OK) return fs;
     for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
     return WIND_OK;
   }
@@ -1397,10 +1402,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     slice_units = std::max<int64_t>(slice_units, grid);  // a burst keeps the whole grid busy
     unsigned long long* t0 = ctx->stamps + slot;
     p.ns_per_byte = 0.f;
-    // a burst-paced op's last pace kernel (after every slice, in stream order) frees the
-    // slot; a stepped op's last layer publication does (op_layer_published)
-    uint32_t* const done_word = p.done_word;
-    if (!step) p.done_word = nullptr;
+
     static PFN_waitValue32 wait_fn = driver_fn<PFN_waitValue32>("cuStreamWaitValue32");
     if (step && !wait_fn) return fail(WIND_ERR_CUDA, "cuStreamWaitValue32 entry point unavailable");
     int launches = 0;
@@ -1426,20 +1428,23 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
       // hold the stream until the schedule reaches the bytes moved so far (after the last
       // slice too: the op then ends when its rate says, as the in-kernel pacer's ops do)
       const double done = payload * static_cast<double>(p.unit_hi) / static_cast<double>(p.total_units);
-      const bool last = p.unit_hi == p.total_units;
-      WKV_CUDA(launch_pace(t0, static_cast<uint64_t>(done * 1e3 / t.rate_mbps), 0, s,
-                           last ? done_word : nullptr, p.op_seq), "pace kernel launch");
+      WKV_CUDA(launch_pace(t0, static_cast<uint64_t>(done * 1e3 / t.rate_mbps), 0, s), "pace kernel launch");
       ++launches;
     }
     g_launches += launches;
+    if ((st = finish_slot(ctx, sl, s)) != WIND_OK) return st;
     for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
     return WIND_OK;
   }
   // rate limit: each of the `grid` CTAs gets rate / grid; ns per payload byte per CTA
   p.ns_per_byte = t.rate_mbps > 0 ? static_cast<float>(grid * 1e3 / t.rate_mbps) : 0.f;
   cudaError_t e = launch_copy(p, kernel, static_cast<int>(grid), s, pdl_enabled());
-  if (e != cudaSuccess) return cuda_fail(e, "copy kernel launch");
+  if (e != cudaSuccess) {
+    release_slot(ctx, sl);  // nothing of this op was enqueued (a debug check is harmless)
+    return cuda_fail(e, "copy kernel launch");
+  }
   g_launches += 1;
+  if ((st = finish_slot(ctx, sl, s)) != WIND_OK) return st;
   for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
   return WIND_OK;
 }

@@ -12,13 +12,12 @@ namespace wkv {
 
 // Per-op, per-layer CTA-arrival counters on each executing device (A5): an op owns one slot
 // of WIND_KV_MAX_LAYERS counters; the arrival completing a layer's units resets its counter.
-// Eager ops take slots [0, kEagerSlots): a slot is handed out again only once its last op has
-// marked it done (the op's final layer publication writes the op's sequence number into a
-// mapped host word) or to the next op of the SAME stream (stream order: that op cannot touch
-// the slot before the previous one completed).  So a long-pending op (a stepped migration
-// waiting on decode steps, an op queued behind a layer_wait) keeps its slot however many ops
-// other streams run meanwhile.  Ops captured into a CUDA graph take slots [kEagerSlots,
-// kCounterSlots) round robin (a replay cannot report completion to the host).
+// Eager ops take slots [0, kEagerSlots) (wind_kv.cpp take_slot): the slot of their stream's
+// previous op (stream order keeps the two apart), else a slot whose last op has completed
+// (a host event recorded after every eager op; no device-side bookkeeping).  So a
+// long-pending op (a stepped migration waiting on decode steps, an op queued behind a
+// layer_wait) keeps its slot however many ops other streams run meanwhile.  Ops captured
+// into a CUDA graph take slots [kEagerSlots, kCounterSlots) round robin.
 constexpr int kEagerSlots = 512;    // streams with ops in flight at once, per device
 constexpr int kGraphSlots = 512;    // captured ops executing concurrently, per device
 constexpr int kCounterSlots = kEagerSlots + kGraphSlots;  // 4 MiB of counters per device
@@ -57,11 +56,6 @@ struct Params {
                               // slices of [0, total_units) on one counter slot)
   int32_t first_slice;        // 1: this launch also bumps the untouched layers' flags
   uint32_t* counters;         // this op's counter slot, [hi - lo]
-  uint32_t* op_layers;        // this slot's count of published layers (reset when it reaches
-                              // n_layers)
-  uint32_t* done_word;        // eager ops: mapped host word; the op's last layer publication
-                              // stores op_seq there (slot free).  NULL: not tracked here
-  uint32_t op_seq;
   const int32_t* abort_word;  // debug pools: skip the copy if the device check fired
   int32_t layer_lo, n_layers; // global lo, hi - lo
   int32_t group;              // table entries per unit (>= 1; > 1 only when C < unit)
@@ -88,10 +82,8 @@ enum Kernel { kAuto = 0, kTma = 1, kSimt = 2, kCopyEngine = 3, kStaged = 4 };
 // to every layer flag of every item (release, system scope).
 cudaError_t launch_flag_bump(const Params& p, cudaStream_t s);
 // Copy-engine rate limit: a 1-thread kernel; `first` stamps the op start in *t0, later
-// launches sleep until *t0 + target_ns.  A non-NULL done_word (the op's last pace kernel)
-// then receives op_seq: the op's counter slot is free.
-cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s,
-                        uint32_t* done_word = nullptr, uint32_t op_seq = 0);
+// launches sleep until *t0 + target_ns.
+cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s);
 
 // wind_kv_step_signal: +1 on a consumer's step counter (release, GPU scope), in stream order.
 cudaError_t launch_step_signal(uint32_t* counter, cudaStream_t s);

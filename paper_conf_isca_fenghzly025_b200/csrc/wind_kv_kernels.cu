@@ -363,23 +363,6 @@ __device__ __forceinline__ void bulk_wait_done_n(int n) {
   }
 }
 
-// The op's slot is free: store op_seq into the mapped host word the allocator polls
-// (wind_kv.cpp take_slot).  Caller ordered every use of the slot before this (fence.sys).
-__device__ __forceinline__ void mark_slot_done(const Params& p) {
-  asm volatile("st.relaxed.sys.global.u32 [%0], %1;" ::"l"(p.done_word), "r"(p.op_seq) : "memory");
-}
-
-// A layer of the op was published (its counter reset): the op's n_layers-th publication —
-// in the op's last slice, once every unit is in — marks the slot done.
-__device__ void op_layer_published(const Params& p) {
-  if (!p.done_word) return;
-  fence_gpu();  // this layer's counter reset before the count
-  if (atomicAdd(p.op_layers, 1u) + 1u != static_cast<uint32_t>(p.n_layers)) return;
-  *reinterpret_cast<volatile uint32_t*>(p.op_layers) = 0u;
-  fence_sys();  // every reset of the slot before the host may hand it out again
-  mark_slot_done(p);
-}
-
 // Arrive on global layer `layer` with the `cnt` units of it this CTA moved; the arrival
 // that completes the layer's 2 x units_per_plane units publishes.  Caller has made this
 // CTA's stores of those units complete and ordered before this call.  Scope: when data and
@@ -401,8 +384,7 @@ __device__ void arrive_layer(const Params& p, int32_t layer, uint32_t cnt) {
     fence_gpu();
   for (int j = 0; j < p.n_items; ++j)
     bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (layer - p.layer_lo), p.items[j]);
-  *reinterpret_cast<volatile uint32_t*>(c) = 0u;  // counter reusable
-  op_layer_published(p);
+  *reinterpret_cast<volatile uint32_t*>(c) = 0u;  // slot reusable
 }
 
 // Debug pools whose device table check fired: nothing is copied, but every layer flag of
@@ -412,10 +394,6 @@ __device__ void publish_aborted(const Params& p) {
   for (int32_t l = p.layer_lo; l < p.layer_lo + p.n_layers; ++l)
     for (int j = 0; j < p.n_items; ++j)
       bump_flag(p.items[j].flags + p.items[j].d_flag_lo + (l - p.layer_lo), p.items[j]);
-  if (p.done_word) {  // no counter was touched
-    fence_sys();
-    mark_slot_done(p);
-  }
 }
 
 // ------------------------------------------------------------------- K2: TMA staged
@@ -638,19 +616,13 @@ __global__ void flag_bump_kernel(const __grid_constant__ Params p) {
   for (int j = 0; j < p.n_items; ++j)
     for (int f = threadIdx.x; f < p.items[j].d_layers; f += blockDim.x)
       bump_flag(p.items[j].flags + f, p.items[j]);
-  __syncthreads();
-  if (threadIdx.x == 0 && p.done_word) {  // the op's pace stamp (in its slot) is no longer read
-    fence_sys();
-    mark_slot_done(p);
-  }
 }
 
 // Copy-engine pacing: one thread (no SM resources worth mentioning, so a rate-limited DMA
 // migration stays off the SMs).  The first launch of an op stamps the op's start time in
 // *t0; every later launch sleeps until t0 + target_ns (the schedule of the bytes copied
 // so far), so command overheads are absorbed and the average rate is exact.
-__global__ void pace_kernel(unsigned long long* t0, uint64_t target_ns, int first,
-                            uint32_t* done_word, uint32_t op_seq) {
+__global__ void pace_kernel(unsigned long long* t0, uint64_t target_ns, int first) {
   if (first) {
     *t0 = globaltimer_ns();
     return;
@@ -661,10 +633,6 @@ __global__ void pace_kernel(unsigned long long* t0, uint64_t target_ns, int firs
     const uint64_t d = until - now;
     __nanosleep(d > 1000000 ? 1000000u : static_cast<unsigned>(d));
     now = globaltimer_ns();
-  }
-  if (done_word) {  // a burst-paced op's last pace kernel: its slot (counters, stamp) is free
-    fence_sys();
-    asm volatile("st.relaxed.sys.global.u32 [%0], %1;" ::"l"(done_word), "r"(op_seq) : "memory");
   }
 }
 
@@ -749,9 +717,8 @@ cudaError_t launch_copy(const Params& p, int kernel, int grid, cudaStream_t s, b
   return cudaLaunchKernelEx(&cfg, simt_copy_kernel, p);
 }
 
-cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s,
-                        uint32_t* done_word, uint32_t op_seq) {
-  pace_kernel<<<1, 1, 0, s>>>(t0, target_ns, first, done_word, op_seq);
+cudaError_t launch_pace(unsigned long long* t0, uint64_t target_ns, int first, cudaStream_t s) {
+  pace_kernel<<<1, 1, 0, s>>>(t0, target_ns, first);
   return cudaGetLastError();
 }
 
