@@ -217,8 +217,12 @@ wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind
  *     automatically outside graph capture (inside a capture, order them yourself); they
  *     must be enqueued by one host thread at a time (the pool's events are reused).
  * A host pool's layer flags live in mapped host memory and are updated without PCIe
- * atomics, so ops INTO one host pool must not overlap in time (ops on one stream never
- * do); the host observes swap_out progress by reading the flags. */
+ * atomics, so ops INTO one host pool must not overlap in time.  The library orders them:
+ * an op into a host pool enqueued on another stream than the pool's previous op first
+ * makes its stream wait (cudaStreamWaitEvent, nothing blocks the host) for that op; ops on
+ * one stream are ordered anyway.  Under graph capture this is not done: order captured
+ * ops into one host pool yourself.  The host observes swap_out progress by reading the
+ * flags. */
 wind_status wind_kv_swap_out(const wind_kv_pool* dev, const int32_t* dev_bt,
                              wind_kv_pool* host, const int32_t* host_bt, int32_t n_blocks,
                              void* stream);

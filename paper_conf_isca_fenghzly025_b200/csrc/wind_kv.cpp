@@ -325,6 +325,16 @@ struct wind_kv_pool {
     cudaEvent_t fork = nullptr, done = nullptr, ready[kStageBufs] = {}, freed[kStageBufs] = {};
     bool has_done = false;            // `done` marks the end of the last uncaptured staged op
   } stg;
+  // Host pools: ops INTO the pool update its layer flags by a plain read-modify-write over
+  // PCIe (no PCIe atomics), so two of them must never overlap.  An op enqueued on another
+  // stream than the pool's previous op first waits for that op's event (HostOrder in run_op);
+  // ops on one stream are ordered anyway.  Not applied under graph capture.
+  struct Order {
+    std::mutex mu;
+    cudaEvent_t ev[kMaxDevices] = {};  // recorded after the last op, on its executing device
+    int last_dev = -1;
+    unsigned long long last_sid = 0;
+  } order;
 };
 
 namespace {
@@ -505,6 +515,8 @@ extern "C" wind_status wind_kv_pool_destroy(wind_kv_pool* p) {
     if (p->owns_flags && p->flags) cudaFree(p->flags);
   } else {
     staging_free(p->stg);
+    for (cudaEvent_t e : p->order.ev)
+      if (e) cudaEventDestroy(e);
     if (p->owns_data && p->base) cudaFreeHost(p->base);
     if (p->owns_flags && p->flags) cudaFreeHost(p->flags);
   }
@@ -856,26 +868,79 @@ wind_status check_ce_tables(int32_t src_nb, const OpItem* items, int n_items) {
 // release_slot undoes a take when the op fails before launching.
 struct Slot {
   int index = -1;
-  bool eager = false;
+  bool eager = false;     // false: the stream is capturing (graph slot ring)
   bool prev_used = false;
   unsigned long long sid = 0, prev_owner = 0;
 };
 
-wind_status take_slot(DevCtx* ctx, int exec, cudaStream_t s, Slot* out) {
+// The stream's unique id (0 if unavailable) and whether it is capturing.
+void stream_identity(cudaStream_t s, unsigned long long* sid, bool* capturing) {
   cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
   if (cudaStreamIsCapturing(s, &cap) != cudaSuccess) {
     cudaGetLastError();
     cap = cudaStreamCaptureStatusNone;
   }
-  if (cap != cudaStreamCaptureStatusNone) {  // a replay cannot be tracked here: round robin
+  *capturing = cap != cudaStreamCaptureStatusNone;
+  *sid = 0;
+  if (!*capturing && cudaStreamGetId(s, sid) != cudaSuccess) {
+    cudaGetLastError();
+    *sid = 0;
+  }
+}
+
+// Orders the ops INTO host pools (wind_kv_pool::Order): holds each host destination's lock
+// from the wait to the record, so two threads cannot both slip in behind the same op.
+class HostOrder {
+ public:
+  HostOrder(const OpItem* items, int n_items, cudaStream_t s, unsigned long long sid, bool capturing)
+      : s_(s), sid_(sid) {
+    if (capturing) return;
+    for (int j = 0; j < n_items; ++j)
+      if (items[j].dst->desc.loc == WIND_LOC_HOST &&
+          std::find(pools_.begin(), pools_.end(), items[j].dst) == pools_.end())
+        pools_.push_back(items[j].dst);
+    std::sort(pools_.begin(), pools_.end());  // one lock order for every thread
+    for (wind_kv_pool* h : pools_) h->order.mu.lock();
+  }
+  ~HostOrder() {
+    for (wind_kv_pool* h : pools_) h->order.mu.unlock();
+  }
+  HostOrder(const HostOrder&) = delete;
+  HostOrder& operator=(const HostOrder&) = delete;
+  // Before the op's first enqueue: wait for the previous op into each pool if it was
+  // enqueued on another stream.
+  wind_status wait() {
+    for (wind_kv_pool* h : pools_) {
+      const auto& o = h->order;
+      if (o.last_dev >= 0 && (sid_ == 0 || o.last_sid != sid_))
+        WKV_CUDA(cudaStreamWaitEvent(s_, o.ev[o.last_dev], 0), "cudaStreamWaitEvent(host pool order)");
+    }
+    return WIND_OK;
+  }
+  // After the op's last enqueue (current device = the executing one).
+  wind_status commit(int exec) {
+    for (wind_kv_pool* h : pools_) {
+      auto& o = h->order;
+      if (!o.ev[exec])
+        WKV_CUDA(cudaEventCreateWithFlags(&o.ev[exec], cudaEventDisableTiming), "cudaEventCreate(host pool order)");
+      WKV_CUDA(cudaEventRecord(o.ev[exec], s_), "cudaEventRecord(host pool order)");
+      o.last_dev = exec;
+      o.last_sid = sid_;
+    }
+    return WIND_OK;
+  }
+
+ private:
+  cudaStream_t s_;
+  unsigned long long sid_;
+  std::vector<wind_kv_pool*> pools_;
+};
+
+wind_status take_slot(DevCtx* ctx, int exec, unsigned long long sid, bool capturing, Slot* out) {
+  if (capturing) {  // a replay cannot be tracked here: round robin
     out->index = kEagerSlots + static_cast<int>(ctx->graph_seq.fetch_add(1) % kGraphSlots);
     out->eager = false;
     return WIND_OK;
-  }
-  unsigned long long sid = 0;
-  if (cudaStreamGetId(s, &sid) != cudaSuccess) {
-    cudaGetLastError();
-    sid = 0;
   }
   std::lock_guard<std::mutex> lk(ctx->slot_mu);
   int idx = -1;
@@ -1216,6 +1281,10 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   }
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   DeviceGuard g(exec);
+  unsigned long long sid = 0;
+  bool capturing = false;
+  stream_identity(s, &sid, &capturing);
+  HostOrder order(items, n_items, s, sid, capturing);  // ops into host pools never overlap
 
   if (step) {  // step-aligned slices: device pools (INTRA / PEER), SM kernels, no debug pools
     bool dbg = false;
@@ -1240,9 +1309,10 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     if (!staged)
       return fail(WIND_ERR_UNSUPPORTED, "staged path needs one item, whole chunks, no rate limit, a "
                   "host-readable host table and host-pool staging on device %d", exec);
+    if ((st = order.wait()) != WIND_OK) return st;
     // hidden chunks run the staged kernel tuning (4 x 48 KiB stages)
-    return staged_host_op(src, items[0], lo, hi, s,
-                          t.max_ctas > 0 ? t.max_ctas : staged_hidden_ctas(src->chunk));
+    st = staged_host_op(src, items[0], lo, hi, s, t.max_ctas > 0 ? t.max_ctas : staged_hidden_ctas(src->chunk));
+    return st == WIND_OK ? order.commit(exec) : st;
   }
   const int kernel = t.kernel == kAuto ? (path == WIND_PATH_PEER ? kSimt : kTma) : t.kernel;
   if (kernel == kStaged)
@@ -1321,7 +1391,11 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   if (kernel == kCopyEngine && (st = check_ce_tables(src->desc.n_blocks, items, n_items)) != WIND_OK) return st;
   // the op's counter slot: the last step that may fail without enqueuing anything
   Slot sl;
-  if ((st = take_slot(ctx, exec, s, &sl)) != WIND_OK) return st;
+  if ((st = take_slot(ctx, exec, sid, capturing, &sl)) != WIND_OK) return st;
+  if ((st = order.wait()) != WIND_OK) {
+    release_slot(ctx, sl);
+    return st;
+  }
   const int slot = sl.index;
   p.counters = ctx->counters + static_cast<size_t>(slot) * WIND_KV_MAX_LAYERS;
   p.abort_word = debug ? ctx->err : nullptr;
@@ -1345,8 +1419,10 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   if (kernel == kCopyEngine) {
     st = copy_engine_op(p, src->desc.n_blocks, items, n_items, s, t.rate_mbps);
     const wind_status fs = finish_slot(ctx, sl, s);  // whatever was enqueued holds the slot
+    const wind_status os = order.commit(exec);
     if (st != WIND_OK) return st;
     if (fs != WIND_OK) return fs;
+    if (os != WIND_OK) return os;
     for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
     return WIND_OK;
   }
@@ -1433,6 +1509,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     }
     g_launches += launches;
     if ((st = finish_slot(ctx, sl, s)) != WIND_OK) return st;
+    if ((st = order.commit(exec)) != WIND_OK) return st;
     for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
     return WIND_OK;
   }
@@ -1445,6 +1522,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   }
   g_launches += 1;
   if ((st = finish_slot(ctx, sl, s)) != WIND_OK) return st;
+  if ((st = order.commit(exec)) != WIND_OK) return st;
   for (int j = 0; j < n_items; ++j) items[j].dst->enqueued.fetch_add(1);
   return WIND_OK;
 }

@@ -25,5 +25,5 @@ timeout -s KILL 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 
   --master-port 29533 bench.py --gpus 2 --steps 5 --warmup 3 --a2a-scale 0.125 --config C1 \
   > $O/${T}_multirank2.log 2>&1; echo "multirank2 rc=$?" >> $O/${T}_multirank2.log
 unset WIND_BENCH_ONE_DEVICE WIND_KV_FORCE_PEER_ROUTE
-bash scripts/sanitize.sh > $O/${T}_sanitize_summary.txt 2>&1
+# (compute-sanitizer runs: round-2 evidence in profiles/r02/sanitizer/; the tool is closed on this pool now)
 ls -la $O > $O/${T}_ls.txt

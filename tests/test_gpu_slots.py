@@ -224,3 +224,76 @@ def test_debug_table_checks_on_two_streams_do_not_share_scratch():
         assert O.migrate(s0, g, sbt, want, g, dbt, 0, L) == O.OK
         np.testing.assert_array_equal(p.tensor().cpu().numpy(), want)
         assert p.layer_count(0) == 10
+
+
+def test_ops_into_one_host_pool_from_two_streams_are_serialised():
+    """A host pool's flags are bumped by a plain read-modify-write over PCIe, so ops INTO it
+    must not overlap.  Stream A's swap_out waits behind a host gate; stream B's swap_out into
+    the same host pool (other host slots) must wait for it — B is still pending while A is
+    held — then both land: host pool == oracle, every flag == 2."""
+    L, H, d, bs, eb = 4, 2, 64, 16, 2
+    rng = np.random.default_rng(35)
+    dev = wk.Pool(L, H, d, bs, eb, 32)
+    s0 = rng.integers(0, 256, dev.nbytes, dtype=np.uint8)
+    dev.tensor().copy_(torch.from_numpy(s0))
+    host = wk.Pool(L, H, d, bs, eb, 32, loc="host")
+    host.tensor().zero_()
+    a_dev, a_host = np.array([4, 9, 1], np.int32), np.array([0, 1, 2], np.int32)
+    b_dev, b_host = np.array([30, 2], np.int32), np.array([10, 11], np.int32)
+    # the tables are borrowed until the ops complete: keep them alive
+    ta_dev, ta_host, tb_dev, tb_host = (torch.as_tensor(x, device=DEV) for x in (a_dev, a_host, b_dev, b_host))
+    A, B = raw_streams(2)
+    torch.cuda.synchronize()
+    gate = HostGate(watchdog_s=60)
+    try:
+        wk.layer_wait(gate.pool, 0, 1, stream=A.handle)
+        wk.swap_out(dev, ta_dev, host, ta_host, stream=A.handle)
+        wk.swap_out(dev, tb_dev, host, tb_host, stream=B.handle)
+        time.sleep(0.05)
+        assert not B.query(), "an op into the host pool overtook a pending one from another stream"
+        gate.set(1)
+        A.synchronize()
+        B.synchronize()
+    finally:
+        gate.close()
+        torch.cuda.synchronize()
+    want = np.zeros(host.nbytes, np.uint8)
+    g = geom(L, H, d, bs, eb, 32)
+    assert O.migrate(s0, g, a_dev, want, g, a_host, 0, L) == O.OK
+    assert O.migrate(s0, g, b_dev, want, g, b_host, 0, L) == O.OK
+    np.testing.assert_array_equal(host.tensor().cpu().numpy(), want)
+    assert [host.layer_count(l) for l in range(L)] == [2] * L
+    for s in (A, B):
+        s.destroy()
+
+
+def test_many_swap_outs_into_one_host_pool_from_four_streams():
+    """Four streams each enqueue 30 small swap_outs into one host pool (disjoint host slots)
+    at once: no flag increment is lost (every flag == 120) and the pool equals the oracle."""
+    L, H, d, bs, eb = 3, 1, 64, 16, 2
+    rng = np.random.default_rng(36)
+    dev = wk.Pool(L, H, d, bs, eb, 64)
+    s0 = rng.integers(0, 256, dev.nbytes, dtype=np.uint8)
+    dev.tensor().copy_(torch.from_numpy(s0))
+    host = wk.Pool(L, H, d, bs, eb, 4 * 30, loc="host")
+    host.tensor().zero_()
+    streams = raw_streams(4)
+    ops = []
+    for k in range(4):
+        for i in range(30):
+            ops.append((k, np.array([rng.integers(0, 64)], np.int32), np.array([k * 30 + i], np.int32)))
+    tabs = [(k, torch.as_tensor(sd, device=DEV), torch.as_tensor(hd, device=DEV), sd, hd) for k, sd, hd in ops]
+    torch.cuda.synchronize()
+    for i in range(30):  # interleaved across the four streams
+        for k in range(4):
+            _, tsd, thd, _, _ = tabs[k * 30 + i]
+            wk.swap_out(dev, tsd, host, thd, stream=streams[k].handle)
+    torch.cuda.synchronize()
+    want = np.zeros(host.nbytes, np.uint8)
+    gd, gh = geom(L, H, d, bs, eb, 64), geom(L, H, d, bs, eb, 120)
+    for _, _, _, sd, hd in tabs:
+        assert O.migrate(s0, gd, sd, want, gh, hd, 0, L) == O.OK
+    np.testing.assert_array_equal(host.tensor().cpu().numpy(), want)
+    assert [host.layer_count(l) for l in range(L)] == [120] * L
+    for s in streams:
+        s.destroy()
