@@ -214,8 +214,9 @@ wind_status wind_kv_migrate(const wind_kv_pool* src, const int32_t* src_bt, wind
  *     nothing enqueued), so it must hold its final values when the call is made; inside a
  *     CUDA graph capture its contents are baked into the graph (a replay moves the slots
  *     the table held at capture).  Staged ops on one host pool serialise on its buffers
- *     automatically outside graph capture (inside a capture, order them yourself); they
- *     must be enqueued by one host thread at a time (the pool's events are reused).
+ *     automatically outside graph capture (inside a capture, order them yourself); ops on
+ *     one host pool are enqueued under the pool's lock, so several host threads may issue
+ *     them.
  * A host pool's layer flags live in mapped host memory and are updated without PCIe
  * atomics, so ops INTO one host pool must not overlap in time.  The library orders them:
  * an op into a host pool enqueued on another stream than the pool's previous op first

@@ -889,21 +889,27 @@ void stream_identity(cudaStream_t s, unsigned long long* sid, bool* capturing) {
 }
 
 // Orders the ops INTO host pools (wind_kv_pool::Order): holds each host destination's lock
-// from the wait to the record, so two threads cannot both slip in behind the same op.
+// from the wait to the record, so two threads cannot both slip in behind the same op.  A
+// host SOURCE pool is only locked (its staging buffers and events, used by the staged path,
+// are then enqueued by one thread at a time).
 class HostOrder {
  public:
-  HostOrder(const OpItem* items, int n_items, cudaStream_t s, unsigned long long sid, bool capturing)
+  HostOrder(const wind_kv_pool* src, const OpItem* items, int n_items, cudaStream_t s,
+            unsigned long long sid, bool capturing)
       : s_(s), sid_(sid) {
-    if (capturing) return;
     for (int j = 0; j < n_items; ++j)
-      if (items[j].dst->desc.loc == WIND_LOC_HOST &&
+      if (!capturing && items[j].dst->desc.loc == WIND_LOC_HOST &&
           std::find(pools_.begin(), pools_.end(), items[j].dst) == pools_.end())
         pools_.push_back(items[j].dst);
-    std::sort(pools_.begin(), pools_.end());  // one lock order for every thread
-    for (wind_kv_pool* h : pools_) h->order.mu.lock();
+    locked_ = pools_;
+    wind_kv_pool* hs = const_cast<wind_kv_pool*>(src);
+    if (src->desc.loc == WIND_LOC_HOST && std::find(locked_.begin(), locked_.end(), hs) == locked_.end())
+      locked_.push_back(hs);
+    std::sort(locked_.begin(), locked_.end());  // one lock order for every thread
+    for (wind_kv_pool* h : locked_) h->order.mu.lock();
   }
   ~HostOrder() {
-    for (wind_kv_pool* h : pools_) h->order.mu.unlock();
+    for (wind_kv_pool* h : locked_) h->order.mu.unlock();
   }
   HostOrder(const HostOrder&) = delete;
   HostOrder& operator=(const HostOrder&) = delete;
@@ -933,7 +939,8 @@ class HostOrder {
  private:
   cudaStream_t s_;
   unsigned long long sid_;
-  std::vector<wind_kv_pool*> pools_;
+  std::vector<wind_kv_pool*> pools_;   // host destinations: ordered
+  std::vector<wind_kv_pool*> locked_;  // pools_ plus a host source
 };
 
 wind_status take_slot(DevCtx* ctx, int exec, unsigned long long sid, bool capturing, Slot* out) {
@@ -1284,7 +1291,7 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   unsigned long long sid = 0;
   bool capturing = false;
   stream_identity(s, &sid, &capturing);
-  HostOrder order(items, n_items, s, sid, capturing);  // ops into host pools never overlap
+  HostOrder order(src, items, n_items, s, sid, capturing);  // ops into host pools never overlap
 
   if (step) {  // step-aligned slices: device pools (INTRA / PEER), SM kernels, no debug pools
     bool dbg = false;

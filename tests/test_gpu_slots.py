@@ -297,3 +297,55 @@ def test_many_swap_outs_into_one_host_pool_from_four_streams():
     assert [host.layer_count(l) for l in range(L)] == [120] * L
     for s in streams:
         s.destroy()
+
+
+def test_staged_swaps_on_one_host_pool_from_four_host_threads():
+    """The staged copy-engine path (kernel 4) reuses a host pool's staging buffers and
+    events; ops on one host pool are enqueued under the pool's lock, so four host threads
+    may issue staged swap_ins from one host pool at once (each into its own device pool, on
+    its own stream): every device pool equals the oracle, every flag == 3."""
+    L, H, d, bs, eb = 4, 4, 64, 16, 2
+    rng = np.random.default_rng(37)
+    host = wk.Pool(L, H, d, bs, eb, 64, loc="host")
+    h0 = rng.integers(0, 256, host.nbytes, dtype=np.uint8)
+    host.tensor().copy_(torch.from_numpy(h0))
+    devs = [wk.Pool(L, H, d, bs, eb, 48) for _ in range(4)]
+    for p in devs:
+        p.tensor().zero_()
+    plans = []
+    for k in range(4):
+        ops = []
+        for _ in range(3):
+            hb = rng.permutation(64)[:10].astype(np.int32)   # host side: read on the CPU (pinned)
+            db = rng.permutation(48)[:10].astype(np.int32)
+            ops.append((hb, db, torch.as_tensor(hb).pin_memory(), torch.as_tensor(db, device=DEV)))
+        plans.append((devs[k], raw_streams(1)[0], ops))
+    saved = wk.get_tuning(wk.PATH_HOST)
+    wk.set_tuning(wk.PATH_HOST, kernel=wk.KERNEL_STAGED)
+    errors = []
+    torch.cuda.synchronize()
+
+    def worker(dev, stream, ops):
+        try:
+            for _, _, thb, tdb in ops:
+                wk.swap_in(host, thb, dev, tdb, stream=stream.handle)
+        except Exception as e:  # noqa: BLE001 — reported below
+            errors.append(e)
+    try:
+        threads = [threading.Thread(target=worker, args=pl) for pl in plans]
+        for th in threads:
+            th.start()
+        for th in threads:
+            th.join()
+        torch.cuda.synchronize()
+    finally:
+        wk.set_tuning(wk.PATH_HOST, **saved)
+    assert not errors, errors
+    g_h, g_d = geom(L, H, d, bs, eb, 64), geom(L, H, d, bs, eb, 48)
+    for dev, stream, ops in plans:
+        want = np.zeros(dev.nbytes, np.uint8)
+        for hb, db, _, _ in ops:
+            assert O.migrate(h0, g_h, hb, want, g_d, db, 0, L) == O.OK
+        np.testing.assert_array_equal(dev.tensor().cpu().numpy(), want)
+        assert [dev.layer_count(l) for l in range(L)] == [3] * L
+        stream.destroy()
