@@ -32,8 +32,9 @@
  *     once; an op on a 513th stream fails with WIND_ERR_UNSUPPORTED, nothing enqueued.  A
  *     pending op (e.g. a stepped migration waiting on decode steps) keeps its slot however
  *     many ops other streams run meanwhile.  Ops captured into a CUDA graph take one of
- *     512 separate graph slots round robin: at most 512 captured ops may execute
- *     concurrently on one device.
+ *     512 separate graph slots round robin, fixed at capture: at most 512 captured ops may
+ *     execute concurrently on one device, and a graph must not run concurrently with
+ *     itself (two replays of one captured op would share its slot).
  *   - `cudaStream_t` parameters are passed as `void*` (0 = the legacy default stream) so
  *     the header needs no CUDA include.
  *   - The copy kernels use programmatic dependent launch: each waits for the previous
