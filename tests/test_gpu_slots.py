@@ -349,3 +349,109 @@ def test_staged_swaps_on_one_host_pool_from_four_host_threads():
         np.testing.assert_array_equal(dev.tensor().cpu().numpy(), want)
         assert [dev.layer_count(l) for l in range(L)] == [3] * L
         stream.destroy()
+
+
+def test_two_streams_of_ops_into_one_device_pool():
+    """R21: concurrent ops into one destination pool with disjoint destination slots.  Two
+    streams enqueue 100 ops each (random layer ranges, interleaved) into one device pool:
+    the pool equals the oracle (the ops commute: disjoint slots) and every layer flag counts
+    all 200 ops (an op bumps every destination layer once, R23)."""
+    L, H, d, bs, eb = 6, 2, 64, 16, 2
+    rng = np.random.default_rng(38)
+    src = wk.Pool(L, H, d, bs, eb, 64)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    dst = wk.Pool(L, H, d, bs, eb, 400)
+    dst.tensor().zero_()
+    A, B = raw_streams(2)
+    ops = []
+    slots = rng.permutation(400).astype(np.int32)
+    for i in range(200):
+        sb = rng.permutation(64)[:2].astype(np.int32)
+        db = slots[2 * i:2 * i + 2].copy()
+        lo = int(rng.integers(0, L))
+        hi = int(rng.integers(lo + 1, L + 1))
+        ops.append((sb, db, lo, hi, torch.as_tensor(sb, device=DEV), torch.as_tensor(db, device=DEV)))
+    torch.cuda.synchronize()
+    for i, (_, _, lo, hi, ts, td) in enumerate(ops):
+        wk.migrate(src, ts, dst, td, layer_lo=lo, layer_hi=hi, stream=(A if i % 2 else B).handle)
+    torch.cuda.synchronize()
+    want = np.zeros(dst.nbytes, np.uint8)
+    gs, gd = geom(L, H, d, bs, eb, 64), geom(L, H, d, bs, eb, 400)
+    for sb, db, lo, hi, _, _ in ops:
+        assert O.migrate(s0, gs, sb, want, gd, db, lo, hi) == O.OK
+    np.testing.assert_array_equal(dst.tensor().cpu().numpy(), want)
+    assert dst.layer_ticket() == 200 and [dst.layer_count(l) for l in range(L)] == [200] * L
+    for s in (A, B):
+        s.destroy()
+
+
+def test_stepped_op_across_the_step_counter_wrap():
+    """wind_kv.h: slice k of a stepped op is released when the step counter reaches
+    first_step + k, 'wrap-safe' (cuStreamWaitValue32 GEQ compares (int32)(*addr - value)).
+    Steps 2^32-2, 2^32-1, 0, 1, ... straddle the uint32 wrap: slices stay blocked until
+    their step, then all land (whole pool == oracle, one flag bump per layer).  The gate is a
+    host-mapped word; its watchdog alternates two release values so a wrong comparison
+    cannot hang the suite."""
+    L, H, d, bs, eb = 8, 8, 128, 16, 2  # 32 KiB chunks
+    nb, n = 48, 40
+    rng = np.random.default_rng(39)
+    src, dst = wk.Pool(L, H, d, bs, eb, nb), wk.Pool(L, H, d, bs, eb, nb)
+    s0 = rng.integers(0, 256, src.nbytes, dtype=np.uint8)
+    d0 = rng.integers(0, 256, dst.nbytes, dtype=np.uint8)
+    src.tensor().copy_(torch.from_numpy(s0))
+    dst.tensor().copy_(torch.from_numpy(d0))
+    sbt = rng.permutation(nb)[:n].astype(np.int32)
+    dbt = rng.permutation(nb)[:n].astype(np.int32)
+    ts, td = torch.as_tensor(sbt, device=DEV), torch.as_tensor(dbt, device=DEV)
+    word_pool = wk.Pool(1, 1, 64, 16, 2, 1, loc="host")
+    word = ct.c_uint32.from_address(word_pool.flags_ptr)
+    first = (1 << 32) - 2
+    word.value = first - 1
+    stop = threading.Event()
+
+    def watchdog():
+        if stop.wait(30):
+            return
+        for i in range(400):  # release under either comparison, alternately
+            word.value = 0xFFFFFFFF if i % 2 else (1 << 20)
+            time.sleep(0.025)
+    wd = threading.Thread(target=watchdog, daemon=True)
+    wd.start()
+    mig = raw_streams(1)[0]
+    torch.cuda.synchronize()
+    try:
+        n0 = wk.launch_count()
+        payload = 2 * L * n * src.chunk_bytes
+        wk.migrate_stepped(src, ts, dst, td, word_pool.flags_ptr, first_step=first,
+                           bytes_per_step=payload // 6 + 1, stream=mig.handle)
+        slices = wk.launch_count() - n0
+        assert slices >= 4
+        time.sleep(0.05)
+        assert not mig.query(), "released before its first step"
+        for k in range(slices - 1):  # steps first .. first + slices - 2 (crossing 2^32)
+            word.value = (first + k) & 0xFFFFFFFF
+            time.sleep(0.05)
+            assert not mig.query(), f"last slice released at step {k} of {slices}"
+        word.value = (first + slices - 1) & 0xFFFFFFFF
+        t_end = time.time() + 10
+        while not mig.query() and time.time() < t_end:
+            time.sleep(0.01)
+        assert mig.query(), "the last slice was not released at its step"
+    finally:
+        # whatever happened above, release every slice under either comparison before
+        # anything synchronises (bounded), then stop the watchdog
+        t_end = time.time() + 20
+        i = 0
+        while not mig.query() and time.time() < t_end:
+            word.value = 0xFFFFFFFF if i % 2 else (1 << 20)
+            i += 1
+            time.sleep(0.025)
+        stop.set()
+        torch.cuda.synchronize()
+    want = d0.copy()
+    g = geom(L, H, d, bs, eb, nb)
+    assert O.migrate(s0, g, sbt, want, g, dbt, 0, L) == O.OK
+    np.testing.assert_array_equal(dst.tensor().cpu().numpy(), want)
+    assert [dst.layer_count(l) for l in range(L)] == [1] * L
+    mig.destroy()
