@@ -164,9 +164,12 @@ wind_status wind_kv_pool_import(const wind_kv_ipc_handle* handle, int32_t local_
  *     unmodified until the op completes on `stream` (the cudaMemcpyAsync contract).
  *   Table contract (R4, R5): entries in range, dst_bt pairwise distinct, and if src and
  *     dst are the same pool, dst_bt[i] == src_bt[j] only for i == j.  Duplicate sources
- *     (fan-out) are allowed.  Release builds do not check table CONTENT on the hot path
- *     (use wind_kv_validate, or WIND_POOL_DEBUG pools); violating it leaves dst undefined
- *     in the affected chunks, never memory outside the two pools' tables' slots.
+ *     (fan-out) are allowed.  Release builds do not CHECK table content on the hot path
+ *     (use wind_kv_validate, or WIND_POOL_DEBUG pools), but they never touch memory
+ *     outside the pools: an entry outside [0, NB) of its pool is skipped (none of its bytes
+ *     read or written; in a fan-out batch, an entry out of range in any destination is
+ *     skipped for all), and the op still publishes every layer flag.  Duplicate or
+ *     aliasing destinations leave the affected chunks of dst undefined.
  *   Executing device: src's device if src is a device pool (its own, or the device an
  *     imported src was mapped into), else dst's.  `stream` must belong to it
  *     (INVALID_ARG otherwise).  Cross-device ops push over NVLink peer stores (or pull
