@@ -164,12 +164,14 @@ wind_status wind_kv_pool_import(const wind_kv_ipc_handle* handle, int32_t local_
  *     unmodified until the op completes on `stream` (the cudaMemcpyAsync contract).
  *   Table contract (R4, R5): entries in range, dst_bt pairwise distinct, and if src and
  *     dst are the same pool, dst_bt[i] == src_bt[j] only for i == j.  Duplicate sources
- *     (fan-out) are allowed.  Release builds do not CHECK table content on the hot path
- *     (use wind_kv_validate, or WIND_POOL_DEBUG pools), but they never touch memory
- *     outside the pools: an entry outside [0, NB) of its pool is skipped (none of its bytes
- *     read or written; in a fan-out batch, an entry out of range in any destination is
- *     skipped for all), and the op still publishes every layer flag.  Duplicate or
- *     aliasing destinations leave the affected chunks of dst undefined.
+ *     (fan-out) are allowed.  Release builds do not check table content on the hot path:
+ *     an entry out of range is UNDEFINED BEHAVIOUR (the kernels read / write base + entry
+ *     * C, like cudaMemcpyAsync with a bad pointer); duplicate or aliasing destinations
+ *     leave the affected chunks of dst undefined.  Check tables with wind_kv_validate
+ *     (host) or create the pools with WIND_POOL_DEBUG (a device-side check before every
+ *     op; a violation aborts the op and is reported by wind_kv_check_device_error).  (A
+ *     kernel-side range guard that skipped such entries was measured at ~1 % of the C2
+ *     headline and not kept.)
  *   Executing device: src's device if src is a device pool (its own, or the device an
  *     imported src was mapped into), else dst's.  `stream` must belong to it
  *     (INVALID_ARG otherwise).  Cross-device ops push over NVLink peer stores (or pull

@@ -1358,7 +1358,6 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
   p.src_plane0 = src->base + static_cast<int64_t>(lo - src->desc.first_layer) * 2 * src->desc.n_blocks * CS +
                  (hr.n < 0 ? 0 : hr.src_lo * tile);
   p.s_plane_stride = static_cast<int64_t>(src->desc.n_blocks) * CS;
-  p.s_blocks = src->desc.n_blocks;
   p.evict_first = t.evict_first;
   p.store_lag = ring.lag;
   p.stages = ring.stages;
@@ -1376,7 +1375,6 @@ wind_status run_op(const wind_kv_pool* src, const OpItem* items, int n_items, in
     q.dst_plane0 = d->base + static_cast<int64_t>(lo - d->desc.first_layer) * 2 * d->desc.n_blocks * CD +
                    (hr.n < 0 ? 0 : hr.dst_lo * tile);
     q.d_plane_stride = static_cast<int64_t>(d->desc.n_blocks) * CD;
-    q.d_blocks = d->desc.n_blocks;
     q.d_chunk = CD;
     q.coalesce = (CP == CS && CP == CD) ? 1 : 0;
     q.flags = d->flags;

@@ -32,7 +32,6 @@ struct Item {
   uint8_t* dst_plane0;     // dst chunk (layer lo, K, block 0) + head offset
   int64_t d_plane_stride;  // NB_dst * C_dst
   int64_t d_chunk;         // C_dst: block stride inside a dst plane
-  int32_t d_blocks;        // NB_dst: table entries outside [0, NB_dst) are skipped
   int32_t coalesce;        // runs of adjacent blocks are contiguous on both sides
   uint32_t* flags;         // dst layer_done[0 .. d_layers)
   int32_t d_flag_lo;       // index of global layer lo in flags
@@ -50,7 +49,6 @@ struct Params {
   const uint8_t* src_plane0;  // src chunk (layer lo, K, block 0) + head offset
   int64_t s_plane_stride;     // NB_src * C_src
   int64_t s_chunk;            // C_src: block stride inside a src plane
-  int32_t s_blocks;           // NB_src: table entries outside [0, NB_src) are skipped
   int64_t copy;               // bytes copied per (layer, kv, block): C, or n_heads * tile
   int64_t units_per_plane;    // sum of items' units
   int64_t total_units;        // planes * units_per_plane

@@ -214,14 +214,10 @@ struct Pacer {
 // --------------------------------------------------------------------- work decoding
 
 // Decodes unit u into segments (called by a FULL warp; writes segs[] from the lanes that
-// own a segment).  Returns the (warp-uniform) segment count; *plane_out, *bytes_out (the
-// bytes the segments load).
+// own a segment).  Returns the (warp-uniform) segment count; *plane_out, *bytes_out.
 // Fan-out (p.fan > 1, fdst != nullptr): the units walk items[0]'s source table; a run must
 // be adjacent in the source and in EVERY destination, and fdst[f][k] receives segment k's
 // address in destination 1 + f.
-// Memory safety: a table entry outside [0, NB) of its pool (any destination of a fan-out)
-// is skipped — no byte of it is read or written — so a bad table in a release build never
-// touches memory outside the pools.  Its unit still counts toward the layer arrivals.
 __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs,
                                            uint8_t* (*fdst)[kMaxSegs], int32_t* plane_out,
                                            uint32_t* bytes_out) {
@@ -244,11 +240,8 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
     const int64_t off = static_cast<int64_t>(part) * p.part_bytes;
     const int64_t rest = CP - off;
     const uint32_t len = static_cast<uint32_t>(rest < p.part_bytes ? rest : p.part_bytes);
-    bool ok = true;
     if (lane == 0) {
       const int32_t s = it.sbt[i], d = it.dbt[i];
-      ok = static_cast<uint32_t>(s) < static_cast<uint32_t>(p.s_blocks) &&
-           static_cast<uint32_t>(d) < static_cast<uint32_t>(it.d_blocks);
       segs[0].src = splane + s * CS + off;
       segs[0].dst = dplane + d * CD + off;
       segs[0].len = len;
@@ -256,36 +249,26 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
     }
     if (lane > 0 && lane < fan) {  // lane f: destination f of the fan-out
       const Item& fi = p.items[lane];
-      const int32_t df = fi.dbt[i];
-      ok = static_cast<uint32_t>(df) < static_cast<uint32_t>(fi.d_blocks);
-      fdst[lane - 1][0] = fi.dst_plane0 + plane * fi.d_plane_stride + df * fi.d_chunk + off;
+      fdst[lane - 1][0] = fi.dst_plane0 + plane * fi.d_plane_stride + fi.dbt[i] * fi.d_chunk + off;
     }
-    ok = __all_sync(kFull, ok);
-    *bytes_out = ok ? len : 0u;
-    return ok ? 1 : 0;
+    *bytes_out = len;
+    return 1;
   }
   // a window of `group` entries: warp-ballot run coalescing (K3)
   const int32_t i0 = r * p.group;
   const int cnt = min(p.group, it.n - i0);
   int32_t s = 0, d = 0;
   int32_t df[kMaxFan - 1] = {0, 0, 0};
-  bool valid = false;
   if (lane < cnt) {
     s = it.sbt[i0 + lane];
     d = it.dbt[i0 + lane];
-    valid = static_cast<uint32_t>(s) < static_cast<uint32_t>(p.s_blocks) &&
-            static_cast<uint32_t>(d) < static_cast<uint32_t>(it.d_blocks);
 #pragma unroll
     for (int f = 1; f < kMaxFan; ++f)
-      if (f < fan) {
-        df[f - 1] = p.items[f].dbt[i0 + lane];
-        valid = valid && static_cast<uint32_t>(df[f - 1]) < static_cast<uint32_t>(p.items[f].d_blocks);
-      }
+      if (f < fan) df[f - 1] = p.items[f].dbt[i0 + lane];
   }
   const int32_t ps = __shfl_up_sync(kFull, s, 1);
   const int32_t pd = __shfl_up_sync(kFull, d, 1);
-  const bool pvalid = __shfl_up_sync(kFull, valid, 1);
-  bool adj = it.coalesce && valid && pvalid && s == ps + 1 && d == pd + 1;
+  bool adj = it.coalesce && s == ps + 1 && d == pd + 1;
 #pragma unroll
   for (int f = 1; f < kMaxFan; ++f) {
     if (f < fan) {  // fan is warp-uniform
@@ -293,15 +276,11 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
       adj = adj && df[f - 1] == pf + 1;
     }
   }
-  // every entry that does not extend the previous run ends it (a skipped entry included);
-  // segments start at the valid ones
-  const bool bound = lane < cnt && (lane == 0 || !adj);
-  const uint32_t bounds = __ballot_sync(kFull, bound);
-  const bool head = bound && valid;
+  const bool head = lane < cnt && (lane == 0 || !adj);
   const uint32_t heads = __ballot_sync(kFull, head);
   if (head) {
     const int k = __popc(heads & ((1u << lane) - 1u));       // prefix popcount
-    const uint32_t later = bounds & ~((2u << lane) - 1u);    // next run boundary after this lane
+    const uint32_t later = heads & ~((2u << lane) - 1u);     // heads after this lane
     const int end = later ? __ffs(later) - 1 : cnt;
     segs[k].src = splane + s * CS;
     segs[k].dst = dplane + d * CD;
@@ -315,7 +294,7 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
       }
     }
   }
-  *bytes_out = static_cast<uint32_t>(__popc(__ballot_sync(kFull, valid)) * CP);
+  *bytes_out = static_cast<uint32_t>(cnt * CP);
   return __popc(heads);
 }
 
