@@ -218,12 +218,12 @@ struct Pacer {
 // Fan-out (p.fan > 1, fdst != nullptr): the units walk items[0]'s source table; a run must
 // be adjacent in the source and in EVERY destination, and fdst[f][k] receives segment k's
 // address in destination 1 + f.
-__device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs,
-                                           uint8_t* (*fdst)[kMaxSegs], int32_t* plane_out,
-                                           uint32_t* bytes_out) {
+// decode_unit_at takes the unit as (plane, r = its index inside the plane); the TMA producer
+// keeps those incrementally (no 64-bit division per unit on its critical path).
+__device__ __forceinline__ int decode_unit_at(const Params& p, int64_t plane, int32_t r, Seg* segs,
+                                              uint8_t* (*fdst)[kMaxSegs], int32_t* plane_out,
+                                              uint32_t* bytes_out) {
   const int lane = threadIdx.x & 31;
-  const int64_t plane = u / p.units_per_plane;
-  int32_t r = static_cast<int32_t>(u - plane * p.units_per_plane);
   int j = 0;
   if (p.fan <= 1)
     while (j + 1 < p.n_items && r >= p.items[j + 1].unit_base) ++j;
@@ -296,6 +296,14 @@ __device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs
   }
   *bytes_out = static_cast<uint32_t>(cnt * CP);
   return __popc(heads);
+}
+
+__device__ __forceinline__ int decode_unit(const Params& p, int64_t u, Seg* segs,
+                                           uint8_t* (*fdst)[kMaxSegs], int32_t* plane_out,
+                                           uint32_t* bytes_out) {
+  const int64_t plane = u / p.units_per_plane;
+  return decode_unit_at(p, plane, static_cast<int32_t>(u - plane * p.units_per_plane), segs, fdst,
+                        plane_out, bytes_out);
 }
 
 // Adds 1 to a layer flag.  The caller has issued the release fence (fence.acq_rel at
@@ -436,6 +444,11 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
       uend = u0 + per < total ? u0 + per : total;
     }
     Pacer pacer;
+    // unit u as (plane, index inside the plane), advanced by ustep without dividing
+    const int64_t upp = p.units_per_plane;
+    int64_t cur_plane = u0 / upp;
+    int64_t cur_r = u0 - cur_plane * upp;
+    const int64_t step_planes = ustep / upp, step_r = ustep - step_planes * upp;
     int it = 0;
     for (int64_t u = u0;; u += ustep, ++it) {
       const int st = it % S;
@@ -451,7 +464,14 @@ __global__ void __launch_bounds__(64, 1) tma_copy_kernel(const __grid_constant__
       }
       int32_t plane;
       uint32_t bytes;
-      const int nseg = decode_unit(p, u, desc[st].segs, desc[st].fdst, &plane, &bytes);
+      const int nseg = decode_unit_at(p, cur_plane, static_cast<int32_t>(cur_r), desc[st].segs,
+                                      desc[st].fdst, &plane, &bytes);
+      cur_plane += step_planes;
+      cur_r += step_r;
+      if (cur_r >= upp) {
+        cur_r -= upp;
+        ++cur_plane;
+      }
       __syncwarp();
       if (lane != 0) mbar_arrive(&full[st]);
       if (lane == 0) {
